@@ -1,0 +1,306 @@
+"""Pins of the CPU oracle against things other than itself (no GPU needed).
+
+Each test names the PAPER.md passage / DESIGN.md reading it pins and the independent
+evidence used: closed forms, finite differences, invariants, brute force with a
+different algorithm, numerical minimisation of Eq. (2), or a library special case
+(scikit-learn CART boosting for MSE, Python's stable sort for the partition).
+"""
+import numpy as np
+import pytest
+from scipy.optimize import minimize
+
+from gen import gen
+
+
+# ------------------------------------------------------------------ binning (R14)
+
+def test_bin_permutation_closed_form(orc):
+    # x a permutation of 0..n-1 with B | n, n > B: bin(x) = floor(x * B / n)   (R14 rule ii)
+    n, B = 1024, 64
+    rng = np.random.default_rng(0)
+    X = rng.permutation(n).astype(np.float32).reshape(n, 1)
+    cuts, nbins, bins = orc.bin_matrix(X, B)
+    assert nbins[0] == B
+    np.testing.assert_array_equal(bins[0], (X[:, 0].astype(np.int64) * B) // n)
+
+
+def test_bin_few_distinct_is_rank(orc):
+    # <= B distinct values: one bin per distinct value, bin = rank among distinct values (R14 rule i)
+    rng = np.random.default_rng(1)
+    vals = np.sort(rng.normal(size=40)).astype(np.float32)
+    X = rng.choice(vals, size=(3000, 1)).astype(np.float32)
+    cuts, nbins, bins = orc.bin_matrix(X, 64)
+    distinct = np.unique(X[:, 0])
+    assert nbins[0] == len(distinct)
+    np.testing.assert_array_equal(bins[0], np.searchsorted(distinct, X[:, 0]))
+
+
+def test_bin_properties_random(orc):
+    rng = np.random.default_rng(2)
+    n, m, B = 5000, 6, 32
+    X = rng.normal(size=(n, m)).astype(np.float32)
+    X[:, 3] = np.round(X[:, 3] * 3)           # ties
+    X[:, 4] = 7.0                             # constant column -> 1 bin
+    cuts, nbins, bins = orc.bin_matrix(X, B)
+    assert nbins[4] == 1 and np.all(bins[4] == 0)
+    for f in range(m):
+        assert 1 <= nbins[f] <= B
+        order = np.argsort(X[:, f], kind="stable")
+        assert np.all(np.diff(bins[f][order].astype(int)) >= 0)          # monotone in x
+        assert bins[f].max() == nbins[f] - 1
+        c = cuts[f][: nbins[f] - 1]
+        assert np.all(np.diff(c) > 0) and np.all(np.isinf(cuts[f][nbins[f] - 1:]))
+        # bin(x) = #{cuts <= x}, checked with numpy's searchsorted (right side)
+        np.testing.assert_array_equal(bins[f], np.searchsorted(c, X[:, f], side="right"))
+    # distinct continuous values: every bin holds >= floor(n/B) rows
+    counts = np.bincount(bins[0], minlength=nbins[0])
+    assert counts.min() >= n // B
+
+
+def test_bin_mnist_shaped_column(orc):
+    # C2 column shape: 81% zeros, rest integers 1..255 -> rule (i), 256 bins, hot bin 0 (DESIGN.md Inputs)
+    w = gen.WORKLOADS["C2"]
+    X = gen.features_host(w, 0, 60000, 0, 2)
+    cuts, nbins, bins = orc.bin_matrix(X, 256)
+    assert list(nbins) == [256, 256]
+    frac0 = np.mean(bins[0] == 0)
+    assert 0.79 < frac0 < 0.83
+
+
+# ------------------------------------------------------------------- gradients
+
+def _mse_loss(y, p):
+    return np.sum((p - y) ** 2)
+
+
+def _ce_loss(y, p):
+    z = p - p.max()
+    return -np.sum(y * (z - np.log(np.sum(np.exp(z)))))
+
+
+@pytest.mark.parametrize("loss", [0, 1])
+def test_grad_finite_differences(orc, loss):
+    # g = dl/dyhat, h = d2l/dyhat_k^2, checked by central differences of the loss itself
+    rng = np.random.default_rng(3)
+    n, d = 7, 5
+    if loss == 0:
+        y = rng.normal(size=(n, d)); f = _mse_loss
+    else:
+        y = np.eye(d)[rng.integers(0, d, n)]; f = _ce_loss
+    p = rng.normal(size=(n, d))
+    g, h = orc.grad(loss, y, p)
+    eps = 1e-4
+    for i in range(n):
+        for k in range(d):
+            e = np.zeros(d); e[k] = eps
+            fp, f0, fm = f(y[i], p[i] + e), f(y[i], p[i]), f(y[i], p[i] - e)
+            assert abs((fp - fm) / (2 * eps) - g[i, k]) < 1e-7 * max(1, abs(g[i, k]))
+            assert abs((fp - 2 * f0 + fm) / eps ** 2 - h[i, k]) < 2e-4
+
+
+def test_softmax_invariants(orc):
+    rng = np.random.default_rng(4)
+    n, d = 500, 10
+    y = np.eye(d)[rng.integers(0, d, n)]
+    p = rng.normal(scale=3, size=(n, d))
+    g, h = orc.grad(1, y, p)
+    assert np.max(np.abs(g.sum(axis=1))) < 1e-14            # sum_k (p_k - y_k) = 0
+    assert np.all(h > 0) and np.all(h <= 0.25)
+
+
+# ------------------------------------------------------------------ histograms
+
+def _tiny(seed, n=300, m=5, d=3, B=16, loss=1):
+    rng = np.random.default_rng(seed)
+    X = rng.normal(size=(n, m)).astype(np.float32)
+    X[:, 1] = rng.integers(0, 6, n)
+    cuts, nbins, bins = oracle_bin_cache(X, B)
+    if loss == 1:
+        y = np.eye(d)[rng.integers(0, d, n)]
+    else:
+        y = rng.normal(size=(n, d))
+    p = rng.normal(size=(n, d))
+    return X, bins, nbins, y, p
+
+
+def oracle_bin_cache(X, B):
+    from oracle import oracle
+    return oracle.bin_matrix(X, B)
+
+
+def test_hist_matches_numpy_scatter_and_invariants(orc):
+    X, bins, nbins, y, p = _tiny(5)
+    g, h = orc.grad(1, y, p)
+    rows = np.random.default_rng(6).permutation(len(X))[:211].astype(np.int32)
+    HG, HH, CNT = orc.build_hist(bins, 16, g, h, rows)
+    m, B, d = HG.shape
+    for f in range(m):
+        ref = np.zeros((B, d)); np.add.at(ref, bins[f][rows], g[rows])       # library scatter-add
+        np.testing.assert_allclose(HG[f], ref, rtol=0, atol=1e-12)
+        np.testing.assert_array_equal(CNT[f], np.bincount(bins[f][rows], minlength=B))
+        np.testing.assert_allclose(HG[f].sum(0), g[rows].sum(0), atol=1e-12)  # sum over bins = node G
+        np.testing.assert_allclose(HH[f].sum(0), h[rows].sum(0), atol=1e-12)
+        assert CNT[f].sum() == len(rows)
+        # softmax: sum_k HG[f][b][k] = 0 for every bin
+        assert np.max(np.abs(HG[f].sum(1))) < 1e-12
+
+
+def test_hist_parent_equals_children_exactly_dyadic(orc):
+    # North-star invariant parent = left + right, bit-exact on dyadic inputs (R24)
+    rng = np.random.default_rng(7)
+    n, m, d, B = 4000, 4, 3, 32
+    X = rng.normal(size=(n, m)).astype(np.float32)
+    cuts, nbins, bins = orc.bin_matrix(X, B)
+    y = np.round(rng.normal(size=(n, d)) * 65536) / 65536
+    g, h = orc.grad(0, y, np.zeros((n, d)))
+    rows = np.arange(n, dtype=np.int32)
+    P = orc.build_hist(bins, B, g, h, rows)
+    left, right = orc.partition(bins, rows, 2, 13)
+    L = orc.build_hist(bins, B, g, h, left)
+    R = orc.build_hist(bins, B, g, h, right)
+    for a, b, c in zip(P, L, R):
+        assert np.array_equal(a, b + c)
+    np.testing.assert_array_equal(P[1], 2.0 * P[2][:, :, None].repeat(d, 2))   # MSE: HH = 2 CNT
+
+
+# ---------------------------------------------------------------- split search
+
+def _exhaustive_best(X, g, h, rows, lam, min_node):
+    """Raw-threshold enumeration: every distinct value v of every feature, left = {x < v},
+    sums straight from the rows, objective from Eq. (2) minimised numerically per side."""
+    best = None
+    for f in range(X.shape[1]):
+        xs = X[rows, f]
+        for v in np.unique(xs)[1:]:
+            L = rows[xs < v]; R = rows[xs >= v]
+            if len(L) < min_node or len(R) < min_node:
+                continue
+            gain = _objective(g[rows], h[rows], lam) - _objective(g[L], h[L], lam) - _objective(g[R], h[R], lam)
+            if best is None or gain > best[0] + 1e-9 * abs(best[0]):
+                best = (gain, f, v)
+    return best
+
+
+def _objective(g, h, lam):
+    """L*(v) of Eq. (2) with diagonal H, by numerical minimisation."""
+    G, H = g.sum(0), h.sum(0)
+    fun = lambda v: float(G @ v + 0.5 * np.sum(H * v * v) + 0.5 * lam * v @ v)
+    jac = lambda v: G + H * v + lam * v
+    r = minimize(fun, np.zeros(len(G)), jac=jac, method="BFGS", options={"gtol": 1e-13, "maxiter": 500})
+    return r.fun
+
+
+@pytest.mark.parametrize("seed,loss", [(10, 1), (11, 0), (12, 1)])
+def test_split_vs_exhaustive_enumeration(orc, seed, loss):
+    X, bins, nbins, y, p = _tiny(seed, n=150, m=4, d=3, B=256, loss=loss)   # B > n: bins = distinct values
+    g, h = orc.grad(loss, y, p)
+    rows = np.arange(len(X), dtype=np.int32)
+    lam, min_node = 1.0, 5
+    HG, HH, CNT = orc.build_hist(bins, 256, g, h, rows)
+    sp = orc.find_split(HG, HH, CNT, nbins, g.sum(0), h.sum(0), len(rows), lam, min_node, want_all=True)
+    gain, f, v = _exhaustive_best(X, g, h, rows, lam, min_node)
+    assert sp["valid"]
+    assert abs(sp["gain"] - gain) <= 1e-7 * abs(gain)
+    # the oracle's winner is the same raw threshold (or ties within the 1e-6 band)
+    cuts, _, _ = orc.bin_matrix(X, 256)
+    thr = cuts[sp["feature"]][sp["bin"]]
+    if (sp["feature"], thr) != (f, v):
+        assert abs(sp["gain"] - gain) <= 1e-6 * abs(gain)
+    # Eq. (3) closed form at every candidate equals the numerically minimised objective difference
+    allg = sp["all_gains"]
+    fb = [(ff, bb) for ff in range(allg.shape[0]) for bb in range(allg.shape[1]) if np.isfinite(allg[ff, bb])]
+    for ff, bb in fb[:: max(1, len(fb) // 12)]:
+        L = rows[bins[ff][rows] <= bb]; R = rows[bins[ff][rows] > bb]
+        ref = _objective(g, h, lam) - _objective(g[L], h[L], lam) - _objective(g[R], h[R], lam)
+        assert abs(allg[ff, bb] - ref) <= 1e-8 * max(1.0, abs(ref))
+
+
+def test_single_output_reduces_to_textbook_gain(orc):
+    # d = 1: GBDT-SO is a special case of GBDT-MO; XGBoost-style gain
+    # 1/2 [GL^2/(HL+l) + GR^2/(HR+l) - G^2/(H+l)] -- compare against the d-output gain of a
+    # problem whose d outputs are identical copies: gain_d = d * gain_1.
+    rng = np.random.default_rng(13)
+    GL, HL, G, H = rng.normal(), rng.uniform(1, 5), rng.normal(), rng.uniform(6, 9)
+    g1 = orc.gain([GL], [HL], [G], [H], 1.0)
+    g4 = orc.gain([GL] * 4, [HL] * 4, [G] * 4, [H] * 4, 1.0)
+    assert abs(g4 - 4 * g1) < 1e-12 * abs(g4)
+
+
+def test_mse_lambda0_gain_is_sse_reduction(orc):
+    # MSE, lambda = 0: Eq. (3) = sum_k SSE reduction (multi-output CART criterion)
+    rng = np.random.default_rng(14)
+    r = rng.normal(size=(60, 3)); mask = rng.random(60) < 0.4
+    g = -2 * r; h = 2 * np.ones_like(r)
+    gain = orc.gain(g[mask].sum(0), h[mask].sum(0), g.sum(0), h.sum(0), 0.0)
+    sse = lambda a: np.sum((a - a.mean(0)) ** 2)
+    assert abs(gain - (sse(r) - sse(r[mask]) - sse(r[~mask]))) < 1e-10 * sse(r)
+
+
+def test_leaf_value_minimises_eq2(orc):
+    rng = np.random.default_rng(15)
+    g = rng.normal(size=(30, 4)); h = rng.uniform(0.1, 1, size=(30, 4)); lam = 0.7
+    v = orc.leaf_value(g.sum(0), h.sum(0), lam, 1.0)
+    G, H = g.sum(0), h.sum(0)
+    r = minimize(lambda x: float(G @ x + 0.5 * np.sum(H * x * x) + 0.5 * lam * x @ x), np.zeros(4),
+                 jac=lambda x: G + H * x + lam * x, method="BFGS", options={"gtol": 1e-14})
+    np.testing.assert_allclose(v, r.x, rtol=1e-7, atol=1e-9)
+
+
+def test_partition_is_stable_sort(orc):
+    X, bins, nbins, y, p = _tiny(16)
+    rows = np.random.default_rng(17).permutation(len(X))[:200].astype(np.int32)
+    left, right = orc.partition(bins, rows, 0, 5)
+    key = (bins[0][rows] > 5).astype(int)
+    ref = rows[np.argsort(key, kind="stable")]                 # library stable sort
+    np.testing.assert_array_equal(np.concatenate([left, right]), ref)
+    assert np.all(bins[0][left] <= 5) and np.all(bins[0][right] > 5)
+
+
+# ------------------------------------------------ whole model: sklearn special case
+
+@pytest.mark.parametrize("D,T", [(4, 5), (3, 3)])
+def test_mse_model_equals_sklearn_residual_trees(orc, D, T):
+    """MSE, lambda = gamma = 0, lr = 1, base 0, min_node 20: T trees of Algorithm 1 =
+    T multi-output CART regressors (max_depth D, min_samples_leaf 20) fitted to residuals
+    on the bin matrix (R1, R2, R4, R9, R10, R11)."""
+    from sklearn.tree import DecisionTreeRegressor
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    y = gen.targets_host(w, X).astype(np.float64)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    res = orc.train(bins, nbins, w.B, y, loss=0, T=T, D=D, lam=0.0, gamma=0.0, lr=1.0, min_node=20)
+    Xb = bins.T.astype(np.float64)
+    pred = np.zeros_like(y)
+    for t in range(T):
+        tree = DecisionTreeRegressor(max_depth=D, min_samples_leaf=20, random_state=0).fit(Xb, y - pred)
+        pred += tree.predict(Xb)
+        root_f = tree.tree_.feature[0]
+        assert res["state"][t][0] == 1 and res["feat"][t][0] == root_f
+        assert res["bin"][t][0] == int(np.floor(tree.tree_.threshold[0]))
+    assert np.max(np.abs(res["pred"] - pred)) < 1e-9
+
+
+def test_train_softmax_invariants(orc):
+    # softmax model (parity unpinned as a whole): structural invariants only
+    w = gen.WORKLOADS["C2"].scaled(n=3000, m=20, T=3, D=3)
+    X = gen.features_host(w, 0, w.n, 0, w.m)
+    y = gen.targets_host(w, X).astype(np.float64)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    res = orc.train(bins, nbins, w.B, y, loss=1, T=3, D=3, lam=1.0, gamma=0.0, lr=1.0, min_node=20)
+    for t in range(3):
+        st, nr, nl = res["state"][t], res["nrows"][t], res["n_left"][t]
+        assert st[0] != 0 and nr[0] == w.n
+        for i in range(len(st)):
+            if st[i] == 1:
+                assert nr[2 * i + 1] == nl[i] and nr[2 * i + 2] == nr[i] - nl[i]
+                assert nl[i] >= 20 and nr[i] - nl[i] >= 20
+        leaves = st == 2
+        assert nr[leaves].sum() == w.n
+        # softmax leaf values sum to ~0 over classes (sum_k G_k = 0, h symmetric-ish not required) -> finite
+        assert np.all(np.isfinite(res["leaf"][t][leaves]))
+    # training reduces the loss
+    p0 = np.zeros_like(y)
+    def ce(p):
+        z = p - p.max(1, keepdims=True)
+        return -np.mean(np.sum(y * (z - np.log(np.exp(z).sum(1, keepdims=True))), 1))
+    assert ce(res["pred"]) < ce(p0)

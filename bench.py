@@ -1,0 +1,396 @@
+"""Benchmark of the GBDT-MO hot path (one training tree = one step) on 1..8 B200s.
+
+Default workload: BASELINE.json configs[4] (C5: n = 2,000,000, m = 4,096, d = 16 outputs,
+256 bins, depth 8, MSE) -- the configuration the metric is quoted on at 1/2/4/8 GPUs.
+Features are partitioned across ranks; every rank replicates y, yhat, g.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5] [--impl ours|reference]
+
+Prints ONE JSON line on rank 0.  `value` = logical histogram rows x outputs per second of the
+whole job: sum over levels of the rows in the nodes searched at that level, times d, divided by
+the device time per tree (max over ranks).  See DESIGN.md "Measurement".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "hist rows*outputs/s (sec/tree alongside)"
+UNIT = "rows*outputs/s"
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="C5")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--graph", action="store_true", help="replay each tree as a CUDA graph (1 GPU)")
+    return ap.parse_args()
+
+
+# --------------------------------------------------------------------------- clocks
+
+class ClockSampler:
+    """nvidia-smi samples during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1])); smax.append(float(f[2])); power.append(float(f[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(smax), "reasons": sorted(reasons),
+                "samples": len(sm), "power_w_max": max(power)}
+
+
+# ---------------------------------------------------------------------------- setup
+
+def shard_range(m, rank, world):
+    return (m * rank) // world, (m * (rank + 1)) // world
+
+
+def built_rows(tree_np, D):
+    """Rows whose histograms were built (root + smaller child of every split with a searched child)."""
+    st, nr, nl = tree_np["node_state"], tree_np["n_rows"], tree_np["n_left"]
+    total = int(nr[0]) if st[0] in (1, 2) and tree_np["_searched"].get(0, False) else 0
+    for h in range(len(st)):
+        if st[h] == 1:
+            lvl = int(np.floor(np.log2(h + 1)))
+            if lvl + 1 >= D:
+                continue
+            l, r = 2 * h + 1, 2 * h + 2
+            if tree_np["_searched"].get(l, False) or tree_np["_searched"].get(r, False):
+                total += int(min(nl[h], nr[h] - nl[h]))
+    return total
+
+
+def annotate_searched(tree_np, D, min_node):
+    st, nr = tree_np["node_state"], tree_np["n_rows"]
+    s = {}
+    for h in range(len(st)):
+        lvl = int(np.floor(np.log2(h + 1)))
+        s[h] = st[h] in (1, 2) and lvl < D and nr[h] >= 2 * min_node
+    tree_np["_searched"] = s
+    return tree_np
+
+
+def host_targets(w):
+    from gen import gen
+    return gen.targets_host(w)
+
+
+# ------------------------------------------------------------------------ CPU oracle
+
+def cpu_oracle_sample(w, feats=128, trees=1):
+    feats = min(feats, w.m)
+    """The oracle as it stands (oracle_train, fp64, OpenMP) on a bounded sample of the workload:
+    all n rows and d outputs, `feats` of the m features, `trees` trees of depth D."""
+    from gen import gen
+    from oracle import oracle
+    cols = np.linspace(0, w.m - 1, feats).astype(np.int64)
+    X = np.empty((w.n, feats), np.float32)
+    for j, c in enumerate(cols):
+        X[:, j] = gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, int(c), 1, w.m)[:, 0]
+    Y = host_targets(w).astype(np.float64)
+    cuts, nbins, bins = oracle.bin_matrix(X, w.B)
+    del X
+    t0 = time.perf_counter()
+    res = oracle.train(bins, nbins, w.B, Y, loss=w.loss, T=trees, D=w.D, lam=w.lam, gamma=w.gamma, lr=w.lr,
+                       min_node=w.min_node)
+    dt = time.perf_counter() - t0
+    ro = 0
+    for t in range(trees):
+        tr = annotate_searched({"node_state": res["state"][t], "n_rows": res["nrows"][t],
+                                "n_left": res["n_left"][t]}, w.D, w.min_node)
+        ro += sum(int(tr["n_rows"][h]) for h, sv in tr["_searched"].items() if sv) * w.d
+    # time scales with the feature count: rate for the full m = ro / (dt * m / feats)
+    value = ro / (dt * w.m / feats)
+    return {"value": value, "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"oracle_train: {trees} tree(s), all {w.n} rows, d={w.d}, depth {w.D}, {feats} of {w.m} "
+                      f"features (evenly spaced); time scaled x{w.m / feats:.0f} to all features",
+            "seconds": dt, "sec_per_tree_full_m": dt / trees * w.m / feats}
+
+
+# ------------------------------------------------------------------------------ main
+
+def main():
+    a = parse()
+    rank, world, local = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1), _env_int("LOCAL_RANK", 0)
+    from gen import gen
+    w = gen.WORKLOADS[a.workload]
+
+    if a.impl == "reference":
+        if rank != 0:
+            return 0
+        cb = cpu_oracle_sample(w)
+        steps = []
+        for _ in range(max(1, min(a.steps, 3))):
+            steps.append(cpu_oracle_sample(w)["value"])
+        val = float(np.median(steps))
+        out = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": a.gpus,
+               "steps": len(steps), "warmup": 1, "ms_per_step": cb["sec_per_tree_full_m"] * 1e3,
+               "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+               "data": "synthetic (seeded counter-based generator, gen/)",
+               "config": {"workload": w.name, "n": w.n, "m": w.m, "d": w.d, "B": w.B, "D": w.D},
+               "cpu_baseline": dict(cb, value=val),
+               "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(out))
+        return 0
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_liupw25_b200 as pkg
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    group = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        group = dist.group.WORLD
+    f0, f1 = shard_range(w.m, rank, world)
+    m_loc = f1 - f0
+    ctx = pkg.Context(local)
+    params = pkg.Params(loss=w.loss, T=a.steps + a.warmup, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
+                        min_node=w.min_node)
+
+    # ---- inputs in HBM (untimed): X shard generated on the device, binned by gbdtmo_bin
+    t_setup = time.perf_counter()
+    Yh = host_targets(w)
+    Y = torch.from_numpy(Yh).to(dev)
+    X = torch.empty((w.n, m_loc), dtype=torch.float32, device=dev)
+    gen.matrix_cuda(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, X.data_ptr(), m_loc,
+                    torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    tb0 = torch.cuda.Event(enable_timing=True); tb1 = torch.cuda.Event(enable_timing=True)
+    tb0.record()
+    ds = pkg.bin_features(ctx, X, w.B, f_begin=f0, m_global=w.m)
+    tb1.record()
+    torch.cuda.synchronize()
+    bin_ms = tb0.elapsed_time(tb1)
+    del X
+    torch.cuda.empty_cache()
+    booster = pkg.Booster(ctx, ds, Y, params, group=group)
+    setup_s = time.perf_counter() - t_setup
+
+    # ---- warm-up
+    for _ in range(a.warmup):
+        booster.step()
+    if a.graph and world == 1:
+        booster.capture()
+    torch.cuda.synchronize()
+    if group is not None:
+        dist.barrier()
+    booster.hist_events.clear()
+
+    # ---- timed region: K trees, device time, max over ranks
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    l0 = ctx.gbdtmo_launch_count()
+    torch.cuda.synchronize()
+    if group is not None:
+        dist.barrier()
+    e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(a.steps):
+        if a.graph and world == 1:
+            booster.step_graph()
+        else:
+            booster.step(time_hist=True)
+    e1.record()
+    torch.cuda.synchronize()
+    if group is not None:
+        dist.barrier()
+    l1 = ctx.gbdtmo_launch_count()
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if group is not None:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    ms_per_tree = ms / a.steps
+
+    # ---- work accounting from the trees' records (after the timed region)
+    trees = [annotate_searched({k: v.cpu().numpy() for k, v in tr.items()}, w.D, w.min_node)
+             for tr in booster.trees[-a.steps:]]
+    ro = sum(sum(int(tr["n_rows"][h]) for h, sv in tr["_searched"].items() if sv) * w.d for tr in trees)
+    rows_built = sum(built_rows(tr, w.D) for tr in trees)
+    value = ro / (ms * 1e-3)
+
+    # ---- dominant kernel: build_hist (zero + k_hist_smem), CUDA events on the launching stream
+    hist_ms = [e0_.elapsed_time(e1_) for (e0_, e1_) in booster.hist_events]
+    hist_launches = len(hist_ms)
+    hist_avg_ms = float(np.sum(hist_ms)) / max(hist_launches, 1)
+    V = booster.p.V
+    updates = rows_built * m_loc * (V + 1)               # per built (row, feature): V channels + count
+    upd_per_launch = updates / max(hist_launches, 1)
+    achieved = upd_per_launch / (hist_avg_ms * 1e-3) if hist_launches else 0.0
+    clock_ghz = 1.965
+    peak = 148 * 16 * clock_ghz * 1e9                     # 32 ATOMS lanes/clk/SM, 2 per update
+    alg_bytes = rows_built * (m_loc + 4 * V + 4)          # bins + q + row id per built row
+    hbm_gbs = alg_bytes / max(hist_launches, 1) / (hist_avg_ms * 1e-3) / 1e9 if hist_launches else 0.0
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except OSError:
+        pass
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "hist_traffic.json")))
+        if prof.get("workload") == w.name:
+            traffic = prof.get("dram_bytes_per_launch")
+    except (OSError, ValueError):
+        pass
+
+    hist_total_ms = float(np.sum(hist_ms))
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": ms_per_tree, "sec_per_tree": ms_per_tree * 1e-3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int64 fixed-point hist / fp64 gains",
+        "data": "synthetic (seeded counter-based generator, gen/); inputs in HBM, 8.2 GB bins >> 126 MB L2 (no flush needed)",
+        "config": {"workload": w.name, "n": w.n, "m": w.m, "d": w.d, "B": w.B, "D": w.D,
+                   "loss": "mse" if w.loss == 0 else "softmax", "parallelism": f"feature-partition x{world}",
+                   "l2": "inputs larger than L2", "graph": bool(a.graph and world == 1)},
+        "hist_share": hist_total_ms / a.steps / ms_per_tree if ms_per_tree else None,
+        "hist_rows_outputs_per_s_built": rows_built * w.d / (hist_total_ms * 1e-3) if hist_ms else None,
+        "bin_ms": bin_ms, "setup_s": setup_s,
+        "roofline": {"bound": "alu", "kernel": "k_hist_smem (+k_zero_build) via gbdtmo_build_hist",
+                     "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tupdate/s",
+                     "frac": achieved / peak if peak else None, "traffic": traffic,
+                     "peak_source": "guide: 32 banks x 4 B/clk/SM shared pipe -> 32 int32 ATOMS lanes/clk/SM, "
+                                    "2 limbs per update, 148 SMs, 1.965 GHz max clock (DESIGN.md Roofline)",
+                     "hbm_view": {"achieved_gbs": hbm_gbs, "peak_gbs": peaks.get("hbm_gbs", 6553.6),
+                                  "frac": hbm_gbs / peaks.get("hbm_gbs", 6553.6)},
+                     "launches": hist_launches, "avg_launch_ms": hist_avg_ms},
+        "clocks": clocks,
+        "gpu_launches": int(l1 - l0),
+    }
+
+    # ---- end to end through the public API with host buffers (H2D inside the timed region)
+    del booster, ds
+    torch.cuda.empty_cache()
+    if not a.no_e2e:
+        out["e2e"] = e2e_run(w, a, rank, world, local, dev, group, f0, f1)
+
+    if group is not None:
+        dist.barrier()
+    if rank == 0:
+        if not a.no_cpu_baseline and world == 1:
+            try:
+                out["cpu_baseline"] = cpu_oracle_sample(w)
+            except Exception as ex:  # report, never fake
+                out["cpu_baseline"] = {"error": repr(ex)}
+        print(json.dumps(out))
+    if group is not None:
+        dist.destroy_process_group()
+    return 0
+
+
+def e2e_run(w, a, rank, world, local, dev, group, f0, f1):
+    """train(): pinned host X shard + y -> H2D -> gbdtmo_bin -> K trees -> D2H of yhat and the trees."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_liupw25_b200 as pkg
+    from gen import gen
+    m_loc = f1 - f0
+    Xh = torch.empty((w.n, m_loc), dtype=torch.float32, pin_memory=True)
+    gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, out=Xh.numpy())
+    Yh = torch.from_numpy(host_targets(w)).pin_memory()
+    ctx = pkg.Context(local)
+    params = pkg.Params(loss=w.loss, T=a.steps, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
+                        min_node=w.min_node)
+    torch.cuda.synchronize()
+    if group is not None:
+        dist.barrier()
+    e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    b = pkg.train(Xh, Yh, params, device=str(dev), ctx=ctx, group=group, f_begin=f0, m_global=w.m)
+    pred_h = torch.empty(b.pred.shape, dtype=b.pred.dtype, pin_memory=True)
+    pred_h.copy_(b.pred, non_blocking=True)
+    model_bytes = 0
+    for tr in b.trees:
+        for k, v in tr.items():
+            model_bytes += v.numel() * v.element_size()
+    model_h = [{k: v.to("cpu", non_blocking=True) for k, v in tr.items()} for tr in b.trees]
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if group is not None:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    ro = 0
+    for tr in model_h:
+        tn = annotate_searched({k: v.numpy() for k, v in tr.items()}, w.D, w.min_node)
+        ro += sum(int(tn["n_rows"][h]) for h, sv in tn["_searched"].items() if sv) * w.d
+    h2d = Xh.numel() * 4 + Yh.numel() * 4
+    d2h = pred_h.numel() * 8 + model_bytes
+    del b
+    torch.cuda.empty_cache()
+    return {"value": ro / (ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d // a.steps,
+            "d2h_bytes_per_step": d2h // a.steps, "ms_total": ms, "trees": a.steps,
+            "what": "pkg.train(host X shard, host y): H2D + gbdtmo_bin + K trees + D2H of yhat and tree records"}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

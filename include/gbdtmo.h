@@ -1,0 +1,243 @@
+/*
+ * gbdtmo.h — C ABI of the B200-native GBDT-MO hot path (libgbdtmo.so, sm_100a).
+ *
+ * Method: Liu, Peng, Wen, "Accelerating Multi-Output GBDTs with GPUs", ICPP'25
+ * (/root/reference/PAPER.md, cited as PAPER.md:<line>).  Notation follows the paper:
+ * n instances, m features, d outputs, B bins, maximum depth
+ * D (Alg. 1's "d", renamed to avoid the clash with #outputs; reading R5),
+ * lambda (l2 on leaves), gamma (split threshold, Alg. 1 input).
+ *
+ * One training tree (Algorithm 1, level-wise reading R6) is driven as
+ *
+ *     gbdtmo_grad                                   (g, h for every instance; tree init)
+ *     for level = 0 .. D-1:
+ *         gbdtmo_build_hist      (level)            (histograms of the nodes marked "build")
+ *         gbdtmo_find_split      (level)            (sibling by subtraction + Eq. (3) + argmax)
+ *         [N > 1: all-reduce MAX of `keys`]
+ *         gbdtmo_split_record    (level)            (owner: left sums + row-direction bitmap)
+ *         [N > 1: all-reduce SUM of `xchg`]
+ *         gbdtmo_partition       (level)            (decisions, stable partition, next level plan)
+ *     gbdtmo_leaf_values
+ *     gbdtmo_update_pred
+ *
+ * Every step is a hand-written CUDA kernel; there is no host fallback.  Nothing in a tree
+ * synchronises with the host: every grid is sized from upper bounds and the per-level node
+ * tables live in device memory (`state`), so a whole tree can be captured in a CUDA graph.
+ *
+ * Conventions
+ *  - Pointers are DEVICE pointers unless marked (host).  The caller owns every buffer; the
+ *    library never allocates device memory except inside gbdtmo_create (nothing) — sizes
+ *    of caller-provided scratch come from the *_bytes queries below.
+ *  - All calls are asynchronous on the context's stream (gbdtmo_set_stream; default: the
+ *    legacy stream 0).  They validate arguments first (GBDTMO_EINVAL, nothing launched),
+ *    then launch and check cudaGetLastError (GBDTMO_ECUDA).  gbdtmo_last_error() returns a
+ *    context-owned message valid until the next call on that context.  No exceptions cross
+ *    the ABI and nothing calls exit/abort.  Outputs of a failed call are unspecified;
+ *    inputs are never written.
+ *  - One context per host thread per device.
+ *  - Fixed point: per tree and per channel c the gradient is stored
+ *    as q = rint(g * 2^30 / P_c), P_c = 2^ceil(log2 max_i |g_ic|) (a power of two, so the
+ *    dequantisation q * scale_c with scale_c = P_c * 2^-30 is exact in fp64).  Histograms
+ *    are exact int64 sums of q; parent = left + right holds exactly and results do not
+ *    depend on the GPU count or the summation order.
+ */
+#ifndef GBDTMO_H
+#define GBDTMO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GBDTMO_ABI_VERSION 1
+
+typedef enum {
+  GBDTMO_OK = 0,
+  GBDTMO_EINVAL = 1,       /* bad argument; nothing launched                              */
+  GBDTMO_ECUDA = 2,        /* CUDA launch / runtime error (message in gbdtmo_last_error)  */
+  GBDTMO_ENOMEM = 3,       /* caller-provided scratch too small                           */
+  GBDTMO_EUNSUPPORTED = 5  /* shape outside the supported envelope (see each call)        */
+} gbdtmo_status;
+
+typedef enum {
+  GBDTMO_LOSS_MSE = 0,     /* l = sum_k (yhat_k - y_k)^2: g = 2(yhat - y), h = 2        */
+  GBDTMO_LOSS_SOFTMAX = 1  /* softmax cross-entropy (reading R12): g = p - y, h = p(1-p) */
+} gbdtmo_loss;
+
+/* Node state in the heap-indexed tree record (root 0, children 2i+1, 2i+2). */
+enum { GBDTMO_NODE_NONE = 0, GBDTMO_NODE_SPLIT = 1, GBDTMO_NODE_LEAF = 2, GBDTMO_NODE_ACTIVE = 3 };
+
+typedef struct gbdtmo_ctx_s* gbdtmo_ctx;
+
+/* Problem description, passed by (host) pointer to every tree call.
+ *   channels V = d (MSE: g only; h = 2 is implicit, H = 2 * count) or 2d (softmax: g then h). */
+typedef struct {
+  int64_t n;          /* instances (rows), 1 <= n < 2^31                                     */
+  int32_t m;          /* features held by this process (its shard), 1 <= m                  */
+  int32_t f_begin;    /* global id of local feature 0 (feature partitioning)   */
+  int32_t m_global;   /* total features over all processes; m_global * B < 2^24             */
+  int32_t d;          /* outputs, 1 <= d <= 1024                                             */
+  int32_t B;          /* maximum bins per feature, 2 <= B <= 256 (bins are uint8)            */
+  int32_t D;          /* maximum depth, 1 <= D <= 12                                         */
+  int32_t loss;       /* gbdtmo_loss                                                         */
+  int32_t min_node;   /* minimum instances per node (reading R4), >= 1         */
+  double lambda;      /* > 0; 0 allowed for tests (H > 0 required then)       */
+  double gamma;       /* >= 0; a node splits iff its best gain > gamma (reading R2, R3)      */
+  double lr;          /* learning rate applied to leaf values (reading R9)     */
+  int64_t ld_bins;    /* row stride of the bins matrix in bytes, multiple of 8, >= m         */
+} gbdtmo_problem;
+
+/* ------------------------------------------------------------------ lifecycle */
+
+int           gbdtmo_abi_version(void);
+gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out /* host */);
+gbdtmo_status gbdtmo_destroy(gbdtmo_ctx ctx);
+gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx ctx, void* cuda_stream /* cudaStream_t */);
+const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
+/* Number of kernels this context has launched so far (for launch accounting). */
+int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
+
+/* ------------------------------------------------------------- size queries (host) */
+
+/* Bytes of the bins buffer: n rows of ld_bins bytes plus 32 bytes of read slack
+ * (the histogram kernel loads 8-byte-aligned windows of up to 32 bytes per row). */
+size_t gbdtmo_bins_bytes(int64_t n, int64_t ld_bins);
+/* Scratch needed by gbdtmo_bin for n rows and m columns. */
+size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B);
+/* Opaque per-tree state (row lists, per-row node ids, heap node tables, launch plans). */
+gbdtmo_status gbdtmo_state_bytes(const gbdtmo_problem* p, size_t* bytes /* host */);
+/* Histogram buffers of one level: hist int64 [2^level][m][B][V], cnt int32 [2^level][m][B]. */
+gbdtmo_status gbdtmo_hist_bytes(const gbdtmo_problem* p, int32_t level, size_t* hist_bytes, size_t* cnt_bytes);
+/* Exchange buffer (int64 elements): 2^(D-1) split records of V+4 words, then ceil(n/64) bitmap words. */
+gbdtmo_status gbdtmo_xchg_count(const gbdtmo_problem* p, int64_t* count /* host */);
+
+/* --------------------------------------------------------------- (a)1 binning */
+
+/* Per-feature quantile binning ("feature-value bin mapping", "cut points"
+ * PAPER.md:166, at most B bins PAPER.md:237, 255; exact rule = reading R14):
+ *   s = sorted column; if it has <= B distinct values the cuts are every distinct value but
+ *   the smallest, else c_j = s[floor(j n / B)], j = 1..B-1, deduplicated, those <= s[0] dropped;
+ *   bin(x) = #{cuts <= x}.
+ * X       float32 row-major, element (i, f) at X[i*ld_x + f]; finite values (-0.0 == +0.0).
+ * bins    uint8, element (i, f) at bins[i*ld_bins + f]; only columns [0, m) are written.
+ * cuts    float32 [m][B-1], ascending, +inf padded.      nbins int32 [m] = #cuts + 1.
+ * ws      scratch of gbdtmo_bin_workspace_bytes(n, m, B) bytes.
+ * Columns are independent: a column slice of a larger matrix may be binned by offsetting
+ * X, bins, cuts and nbins.  EUNSUPPORTED if B > 256. */
+gbdtmo_status gbdtmo_bin(gbdtmo_ctx ctx, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t B,
+                         uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
+                         void* ws, size_t ws_bytes);
+
+/* ------------------------------------------------------------ (a)2 gradients */
+
+/* First/second derivatives per output (softmax reading R12, diagonal
+ * Hessian PAPER.md:96), quantised to fixed point, plus initialisation of the tree state:
+ *   y      float32 [n][d]   targets (softmax: one-hot or any row summing to 1)
+ *   pred   float64 [n][d]   current prediction yhat (sum of previous trees)
+ *   q      int32   [n][V]   out: q[i][c] (MSE: g; softmax: g for c < d, h for c >= d)
+ *   scales float32 [V]      out: dequantisation factor P_c * 2^-30 (a power of two)
+ *   state  gbdtmo_state_bytes(p) bytes, out: root node = all rows (sums of q = exact int64),
+ *          per-row node ids = root, level-0 build plan. */
+gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* y, const double* pred,
+                          int32_t* q, float* scales, void* state);
+
+/* ------------------------------------------------------ (a)3 histogram build */
+
+/* For every node of `level` marked "build" by the plan in `state` (the root at level 0, the
+ * smaller child of each split afterwards, reading R19), for every local feature f, bin b and
+ * channel c:   hist[slot][f][b][c] = sum_{i in node, bin(i,f) = b} q[i][c]   (exact int64),
+ *              cnt [slot][f][b]    = #{i in node : bin(i,f) = b}.
+ * (§3.3; the paper's Alg. 2 body is missing.)
+ * bins uint8 with ld = p->ld_bins and gbdtmo_bins_bytes() of storage; q from gbdtmo_grad;
+ * hist / cnt: this level's buffers (gbdtmo_hist_bytes(level)); slot = node index within the
+ * level (heap id - (2^level - 1)).  Slots not built are left untouched. */
+gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                const uint8_t* bins, const int32_t* q, void* state,
+                                int64_t* hist, int32_t* cnt);
+
+/* ------------------------------------- (a)4 subtraction + (a)5 split search */
+
+/* For every active node of `level`:
+ *   - if marked "derive": hist = parent_hist[parent] - hist[sibling] (and cnt likewise),
+ *     written to its slot when level < D-1 (it is a parent at the next level);
+ *   - for every local feature f and candidate bin b in [0, nbins[f]-2] (left = bins <= b,
+ *     reading R15): G_L, H_L, C_L by prefix sums over bins, valid iff
+ *     C_L >= min_node and C_R >= min_node (R4), gain by Eq. (3) in fp64;
+ *   - keys[slot] = max over candidates with gain > gamma of
+ *       (bits(gain) & ~0xFFFFFF) | (0xFFFFFF - (f_global * B + b))
+ *     (0 if none): larger gain wins, ties -> smallest (f, b) (reading R16); the same key is
+ *     max-reduced across GPUs.
+ * nbins int32 [m] (local features); scales from gbdtmo_grad; keys uint64 [2^level] (out,
+ * every slot written).  parent_hist / parent_cnt: level-1 buffers (ignored at level 0). */
+gbdtmo_status gbdtmo_find_split(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                const int32_t* nbins, const float* scales, void* state,
+                                int64_t* hist, int32_t* cnt,
+                                const int64_t* parent_hist, const int32_t* parent_cnt,
+                                uint64_t* keys);
+
+/* ------------------------------------------------------------ (a)6 exchange */
+
+/* Split records of `level`, written by the process that owns each winning feature
+ * (all-zero elsewhere, so a SUM all-reduce across processes merges them):
+ *   xchg[slot*(V+4) + c]   = G_L sums (int64 fixed point) at the winner, c < V
+ *   xchg[slot*(V+4) + V]   = C_L
+ *   xchg[slot*(V+4) + V+1] = winning global feature + 1 (0: node does not split)
+ *   xchg[slot*(V+4) + V+2] = winning bin
+ *   xchg[slot*(V+4) + V+3] = bits of the fp64 gain
+ *   xchg[2^(D-1)*(V+4) + w] bitmap: bit (i & 63) of word (i >> 6) = 1 iff instance i sits in a
+ *                            splitting node of this level and goes left (bin <= b).
+ * keys: this level's keys after the (optional) MAX all-reduce; scales from gbdtmo_grad;
+ * hist / cnt / parent_hist / parent_cnt as for gbdtmo_find_split (a derived winner's sums are
+ * parent - sibling).  Every xchg word is written. */
+gbdtmo_status gbdtmo_split_record(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                  const uint8_t* bins, const float* scales, void* state,
+                                  const int64_t* hist, const int32_t* cnt,
+                                  const int64_t* parent_hist, const int32_t* parent_cnt,
+                                  const uint64_t* keys, int64_t* xchg);
+
+/* ------------------------------------------------------------ (a)7 partition */
+
+/* Applies the (merged) split records of `level` (Alg. 1 lines 14-17):
+ * nodes with a record split, the others become leaves; the rows of each splitting node are
+ * stably partitioned into left (bit = 1) then right, preserving their order; per-row node ids
+ * move to the children; children get exact sums (left = record, right = parent - left), the
+ * state ACTIVE if level+1 < D and they hold >= 2*min_node rows (else LEAF); the smaller child
+ * (ties: left) is marked "build", the larger "derive" (reading R19); the next level's build
+ * plan is written.  Identical on every process given identical xchg. */
+gbdtmo_status gbdtmo_partition(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level, void* state,
+                               const int64_t* xchg);
+
+/* ------------------------------------------------------------ (a)8, (a)9 */
+
+/* Leaf values: for every heap node in state LEAF,
+ *   leaf[h][k] = -lr * G_k / (H_k + lambda)   (G, H = exact node sums, MSE: H = 2 * count);
+ * other heap nodes get 0.  leaf float64 [2^(D+1)-1][d]. */
+gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* scales,
+                                 void* state, double* leaf);
+
+/* Incremental prediction (rows read their leaf directly, no traversal):
+ *   pred[i][k] += leaf[node_of(i)][k]   for every instance i.   pred float64 [n][d] in/out
+ * (fp64 so that the prediction does not drift from the fp64 definition over many trees). */
+gbdtmo_status gbdtmo_update_pred(gbdtmo_ctx ctx, const gbdtmo_problem* p, const void* state,
+                                 const double* leaf, double* pred);
+
+/* Copy of the tree record (heap-indexed, 2^(D+1)-1 entries each) out of `state`:
+ * node_state (GBDTMO_NODE_*), feature (global id, -1 if none), bin, gain (fp64),
+ * n_rows, n_left.  Any output pointer may be NULL. */
+gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx ctx, const gbdtmo_problem* p, const void* state,
+                                 int32_t* node_state, int32_t* feature, int32_t* bin, double* gain,
+                                 int64_t* n_rows, int64_t* n_left);
+
+/* Copy of the row bookkeeping out of `state` (tests, debugging): the row-index list as seen by
+ * `level` (level = D: after the last partition), int32 [n]; the heap node of every instance,
+ * int32 [n]; and the [begin, end) positions of every heap node in that list, int32 [2^(D+1)-1]
+ * each.  Any output pointer may be NULL. */
+gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx ctx, const gbdtmo_problem* p, const void* state, int32_t level,
+                                 int32_t* rows, int32_t* node_of_row, int32_t* node_begin, int32_t* node_end);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GBDTMO_H */

@@ -1,0 +1,201 @@
+"""Thin ctypes binding of libgbdtmo.so (include/gbdtmo.h): argument marshalling only.
+
+Every function has the C name and forwards plain integers / pointers; tensors are passed by
+their data pointer (``t.data_ptr()``).  A non-OK status raises ``GbdtmoError`` with the
+library's message.  There is no fallback: if the library is missing this module raises on
+import of :func:`lib`.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgbdtmo.so")
+
+OK, EINVAL, ECUDA, ENOMEM, EUNSUPPORTED = 0, 1, 2, 3, 5
+LOSS_MSE, LOSS_SOFTMAX = 0, 1
+NODE_NONE, NODE_SPLIT, NODE_LEAF, NODE_ACTIVE = 0, 1, 2, 3
+
+# Every symbol include/gbdtmo.h declares (checked by tests/test_abi_load.py).
+SYMBOLS = (
+    "gbdtmo_abi_version", "gbdtmo_create", "gbdtmo_destroy", "gbdtmo_set_stream", "gbdtmo_last_error",
+    "gbdtmo_launch_count", "gbdtmo_bins_bytes", "gbdtmo_bin_workspace_bytes", "gbdtmo_state_bytes",
+    "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
+    "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
+    "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export",
+)
+
+
+class GbdtmoError(RuntimeError):
+    pass
+
+
+class Problem(C.Structure):
+    """gbdtmo_problem (include/gbdtmo.h)."""
+    _fields_ = [("n", C.c_int64), ("m", C.c_int32), ("f_begin", C.c_int32), ("m_global", C.c_int32),
+                ("d", C.c_int32), ("B", C.c_int32), ("D", C.c_int32), ("loss", C.c_int32),
+                ("min_node", C.c_int32), ("lambda_", C.c_double), ("gamma", C.c_double), ("lr", C.c_double),
+                ("ld_bins", C.c_int64)]
+
+    @property
+    def V(self):
+        return 2 * self.d if self.loss == LOSS_SOFTMAX else self.d
+
+
+_LIB = None
+
+
+def lib():
+    global _LIB
+    if _LIB is None:
+        if not os.path.exists(LIB_PATH):
+            raise GbdtmoError(f"{LIB_PATH} not built: run `make` or __graft_entry__.build()")
+        L = C.CDLL(LIB_PATH)
+        P, i32, i64, f64, sz = C.c_void_p, C.c_int32, C.c_int64, C.c_double, C.c_size_t
+        PP = C.POINTER(Problem)
+        sig = {
+            "gbdtmo_abi_version": ([], C.c_int),
+            "gbdtmo_create": ([C.c_int, C.POINTER(P)], C.c_int),
+            "gbdtmo_destroy": ([P], C.c_int),
+            "gbdtmo_set_stream": ([P, P], C.c_int),
+            "gbdtmo_last_error": ([P], C.c_char_p),
+            "gbdtmo_launch_count": ([P], i64),
+            "gbdtmo_bins_bytes": ([i64, i64], sz),
+            "gbdtmo_bin_workspace_bytes": ([i64, i32, i32], sz),
+            "gbdtmo_state_bytes": ([PP, C.POINTER(sz)], C.c_int),
+            "gbdtmo_hist_bytes": ([PP, i32, C.POINTER(sz), C.POINTER(sz)], C.c_int),
+            "gbdtmo_xchg_count": ([PP, C.POINTER(i64)], C.c_int),
+            "gbdtmo_bin": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz], C.c_int),
+            "gbdtmo_grad": ([P, PP, P, P, P, P, P], C.c_int),
+            "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P], C.c_int),
+            "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
+            "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
+            "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
+            "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
+        }
+        for name, (args, res) in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _LIB = L
+    return _LIB
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if isinstance(t, int):
+        return t
+    return t.data_ptr()
+
+
+class Context:
+    """Owns one gbdtmo_ctx; methods mirror the C calls (same names without the prefix)."""
+
+    def __init__(self, device: int = 0):
+        self._h = C.c_void_p()
+        st = lib().gbdtmo_create(device, C.byref(self._h))
+        if st != OK:
+            raise GbdtmoError(f"gbdtmo_create(device={device}) failed with status {st}")
+
+    def close(self):
+        if self._h:
+            lib().gbdtmo_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, st, name):
+        if st != OK:
+            msg = lib().gbdtmo_last_error(self._h)
+            raise GbdtmoError(f"{name}: status {st}: {msg.decode() if msg else ''}")
+
+    # lifecycle -------------------------------------------------------------
+    def gbdtmo_set_stream(self, stream_handle: int):
+        self._check(lib().gbdtmo_set_stream(self._h, C.c_void_p(stream_handle)), "gbdtmo_set_stream")
+
+    def gbdtmo_launch_count(self) -> int:
+        return int(lib().gbdtmo_launch_count(self._h))
+
+    # sizes (host) ------------------------------------------------------------
+    @staticmethod
+    def gbdtmo_bins_bytes(n, ld_bins) -> int:
+        return int(lib().gbdtmo_bins_bytes(n, ld_bins))
+
+    @staticmethod
+    def gbdtmo_bin_workspace_bytes(n, m, B) -> int:
+        return int(lib().gbdtmo_bin_workspace_bytes(n, m, B))
+
+    @staticmethod
+    def gbdtmo_state_bytes(p: Problem) -> int:
+        v = C.c_size_t()
+        if lib().gbdtmo_state_bytes(C.byref(p), C.byref(v)) != OK:
+            raise GbdtmoError("gbdtmo_state_bytes: invalid problem")
+        return int(v.value)
+
+    @staticmethod
+    def gbdtmo_hist_bytes(p: Problem, level: int):
+        h, c = C.c_size_t(), C.c_size_t()
+        if lib().gbdtmo_hist_bytes(C.byref(p), level, C.byref(h), C.byref(c)) != OK:
+            raise GbdtmoError("gbdtmo_hist_bytes: invalid problem or level")
+        return int(h.value), int(c.value)
+
+    @staticmethod
+    def gbdtmo_xchg_count(p: Problem) -> int:
+        v = C.c_int64()
+        if lib().gbdtmo_xchg_count(C.byref(p), C.byref(v)) != OK:
+            raise GbdtmoError("gbdtmo_xchg_count: invalid problem")
+        return int(v.value)
+
+    # the hot-path calls --------------------------------------------------------
+    def gbdtmo_bin(self, X, n, m, ld_x, B, bins, ld_bins, cuts, nbins, ws, ws_bytes):
+        self._check(lib().gbdtmo_bin(self._h, _ptr(X), n, m, ld_x, B, _ptr(bins), ld_bins, _ptr(cuts),
+                                     _ptr(nbins), _ptr(ws), ws_bytes), "gbdtmo_bin")
+
+    def gbdtmo_grad(self, p, y, pred, q, scales, state):
+        self._check(lib().gbdtmo_grad(self._h, C.byref(p), _ptr(y), _ptr(pred), _ptr(q), _ptr(scales),
+                                      _ptr(state)), "gbdtmo_grad")
+
+    def gbdtmo_build_hist(self, p, level, bins, q, state, hist, cnt):
+        self._check(lib().gbdtmo_build_hist(self._h, C.byref(p), level, _ptr(bins), _ptr(q), _ptr(state),
+                                            _ptr(hist), _ptr(cnt)), "gbdtmo_build_hist")
+
+    def gbdtmo_find_split(self, p, level, nbins, scales, state, hist, cnt, parent_hist, parent_cnt, keys):
+        self._check(lib().gbdtmo_find_split(self._h, C.byref(p), level, _ptr(nbins), _ptr(scales), _ptr(state),
+                                            _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
+                                            _ptr(keys)), "gbdtmo_find_split")
+
+    def gbdtmo_split_record(self, p, level, bins, scales, state, hist, cnt, parent_hist, parent_cnt, keys, xchg):
+        self._check(lib().gbdtmo_split_record(self._h, C.byref(p), level, _ptr(bins), _ptr(scales), _ptr(state),
+                                              _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
+                                              _ptr(keys), _ptr(xchg)), "gbdtmo_split_record")
+
+    def gbdtmo_partition(self, p, level, state, xchg):
+        self._check(lib().gbdtmo_partition(self._h, C.byref(p), level, _ptr(state), _ptr(xchg)),
+                    "gbdtmo_partition")
+
+    def gbdtmo_leaf_values(self, p, scales, state, leaf):
+        self._check(lib().gbdtmo_leaf_values(self._h, C.byref(p), _ptr(scales), _ptr(state), _ptr(leaf)),
+                    "gbdtmo_leaf_values")
+
+    def gbdtmo_update_pred(self, p, state, leaf, pred):
+        self._check(lib().gbdtmo_update_pred(self._h, C.byref(p), _ptr(state), _ptr(leaf), _ptr(pred)),
+                    "gbdtmo_update_pred")
+
+    def gbdtmo_tree_export(self, p, state, node_state=None, feature=None, bin=None, gain=None, n_rows=None,
+                           n_left=None):
+        self._check(lib().gbdtmo_tree_export(self._h, C.byref(p), _ptr(state), _ptr(node_state), _ptr(feature),
+                                             _ptr(bin), _ptr(gain), _ptr(n_rows), _ptr(n_left)),
+                    "gbdtmo_tree_export")
+
+    def gbdtmo_rows_export(self, p, state, level, rows=None, node_of_row=None, node_begin=None, node_end=None):
+        self._check(lib().gbdtmo_rows_export(self._h, C.byref(p), _ptr(state), level, _ptr(rows), _ptr(node_of_row),
+                                             _ptr(node_begin), _ptr(node_end)), "gbdtmo_rows_export")

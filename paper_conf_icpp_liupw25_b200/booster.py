@@ -1,0 +1,204 @@
+"""Driver of Algorithm 1 over the C ABI — host orchestration only.
+
+Every arithmetic step runs in libgbdtmo.so kernels; this module allocates device buffers
+with torch (plumbing), issues the ABI calls level by level, and — when a process group is
+given — performs the two per-level exchanges of the feature-partitioned multi-GPU scheme
+ with torch.distributed (NCCL): a MAX all-reduce of the packed split keys and
+a SUM all-reduce of the owners' split records + row-direction bitmap.  Nothing in a tree
+waits for the host, so a whole tree can be replayed as one CUDA graph.
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+from typing import Optional
+
+import torch
+
+from . import _abi
+from ._abi import Context, Problem, LOSS_MSE, LOSS_SOFTMAX
+
+
+@dataclasses.dataclass
+class Params:
+    """Training parameters; defaults are the paper's: 100 trees, depth 7,
+    learning rate 1, >= 20 instances per node, 256 bins; lambda = 1, gamma = 0 (readings R1, R2)."""
+    loss: int = LOSS_MSE
+    T: int = 100
+    D: int = 7
+    B: int = 256
+    lam: float = 1.0
+    gamma: float = 0.0
+    lr: float = 1.0
+    min_node: int = 20
+
+
+def _align(x, a):
+    return (x + a - 1) // a * a
+
+
+@dataclasses.dataclass
+class Dataset:
+    """Binned feature shard resident in HBM: bins uint8 [n][ld_bins] (row-major), cuts, nbins."""
+    bins: torch.Tensor          # flat uint8 of gbdtmo_bins_bytes(n, ld_bins)
+    nbins: torch.Tensor         # int32 [m]
+    cuts: torch.Tensor          # float32 [m][B-1]
+    n: int
+    m: int
+    ld_bins: int
+    B: int
+    f_begin: int = 0
+    m_global: int = 0
+
+
+def bin_features(ctx: Context, X: torch.Tensor, B: int, f_begin: int = 0, m_global: Optional[int] = None,
+                 bins_out: Optional[torch.Tensor] = None, ws: Optional[torch.Tensor] = None) -> Dataset:
+    """gbdtmo_bin on a device float32 matrix [n][m] (row stride X.stride(0))."""
+    assert X.is_cuda and X.dtype == torch.float32 and X.stride(1) == 1
+    n, m = X.shape
+    ld = _align(m, 16)
+    nbytes = ctx.gbdtmo_bins_bytes(n, ld)
+    bins = bins_out if bins_out is not None else torch.empty(nbytes, dtype=torch.uint8, device=X.device)
+    cuts = torch.empty((m, B - 1), dtype=torch.float32, device=X.device)
+    nbins = torch.empty(m, dtype=torch.int32, device=X.device)
+    wsb = ctx.gbdtmo_bin_workspace_bytes(n, m, B)
+    if ws is None or ws.numel() < wsb:
+        ws = torch.empty(wsb, dtype=torch.uint8, device=X.device)
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream(X.device).cuda_stream)
+    ctx.gbdtmo_bin(X, n, m, X.stride(0), B, bins, ld, cuts, nbins, ws, wsb)
+    return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m)
+
+
+class Booster:
+    """One GBDT-MO model being trained on one GPU (one feature shard when `group` is given)."""
+
+    def __init__(self, ctx: Context, ds: Dataset, y: torch.Tensor, params: Params,
+                 group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True):
+        self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
+        dev = ds.bins.device
+        self.device = dev
+        n, d = y.shape
+        assert n == ds.n and y.dtype == torch.float32 and y.is_contiguous()
+        self.y = y
+        self.d = d
+        self.p = Problem(n=n, m=ds.m, f_begin=ds.f_begin, m_global=ds.m_global or ds.m, d=d, B=ds.B, D=params.D,
+                         loss=params.loss, min_node=params.min_node, lambda_=params.lam, gamma=params.gamma,
+                         lr=params.lr, ld_bins=ds.ld_bins)
+        V = self.p.V
+        D = params.D
+        self.pred = pred if pred is not None else torch.zeros((n, d), dtype=torch.float64, device=dev)
+        assert self.pred.dtype == torch.float64
+        self.q = torch.empty((n, V), dtype=torch.int32, device=dev)
+        self.scales = torch.empty(V, dtype=torch.float32, device=dev)
+        self.state = torch.empty(ctx.gbdtmo_state_bytes(self.p), dtype=torch.uint8, device=dev)
+        self.hist, self.cnt = [None, None], [None, None]
+        for lvl in (D - 1, D - 2):
+            if lvl < 0:
+                continue
+            hb, cb = ctx.gbdtmo_hist_bytes(self.p, lvl)
+            self.hist[lvl % 2] = torch.empty(hb // 8, dtype=torch.int64, device=dev)
+            self.cnt[lvl % 2] = torch.empty(cb // 4, dtype=torch.int32, device=dev)
+        if self.hist[1] is None:
+            self.hist[1], self.cnt[1] = self.hist[0], self.cnt[0]
+        self.keys = torch.zeros(1 << max(D - 1, 0), dtype=torch.int64, device=dev)
+        self.xchg = torch.zeros(ctx.gbdtmo_xchg_count(self.p), dtype=torch.int64, device=dev)
+        NH = (1 << (D + 1)) - 1
+        self.NH = NH
+        self.leaf = torch.empty((NH, d), dtype=torch.float64, device=dev)
+        self.keep_model = keep_model
+        self.trees = []            # per tree: dict of device tensors (heap-indexed tree record)
+        self._graph = None
+        self.hist_events = []      # optional per-level (start, end) CUDA events around build_hist
+
+    # ------------------------------------------------------------------ one tree
+    def _level(self, lvl: int, time_hist: bool = False):
+        ctx, p = self.ctx, self.p
+        cur, par = lvl % 2, (lvl - 1) % 2
+        ph = self.hist[par] if lvl > 0 else None
+        pc = self.cnt[par] if lvl > 0 else None
+        if time_hist:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+        ctx.gbdtmo_build_hist(p, lvl, self.ds.bins, self.q, self.state, self.hist[cur], self.cnt[cur])
+        if time_hist:
+            e1.record()
+            self.hist_events.append((e0, e1))
+        ctx.gbdtmo_find_split(p, lvl, self.ds.nbins, self.scales, self.state, self.hist[cur], self.cnt[cur],
+                              ph, pc, self.keys)
+        if self.group is not None:
+            torch.distributed.all_reduce(self.keys[: 1 << lvl], op=torch.distributed.ReduceOp.MAX, group=self.group)
+        ctx.gbdtmo_split_record(p, lvl, self.ds.bins, self.scales, self.state, self.hist[cur], self.cnt[cur],
+                                ph, pc, self.keys, self.xchg)
+        if self.group is not None:
+            torch.distributed.all_reduce(self.xchg, op=torch.distributed.ReduceOp.SUM, group=self.group)
+        ctx.gbdtmo_partition(p, lvl, self.state, self.xchg)
+
+    def _tree(self, time_hist: bool = False):
+        ctx, p = self.ctx, self.p
+        ctx.gbdtmo_set_stream(torch.cuda.current_stream(self.device).cuda_stream)
+        ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state)
+        for lvl in range(self.params.D):
+            self._level(lvl, time_hist)
+        ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf)
+        ctx.gbdtmo_update_pred(p, self.state, self.leaf, self.pred)
+
+    def step(self, time_hist: bool = False):
+        """One boosting iteration (one tree) on the current stream; asynchronous."""
+        self._tree(time_hist)
+        if self.keep_model:
+            self.trees.append(self.export())
+
+    def export(self):
+        NH, dev = self.NH, self.device
+        rec = dict(node_state=torch.empty(NH, dtype=torch.int32, device=dev),
+                   feature=torch.empty(NH, dtype=torch.int32, device=dev),
+                   bin=torch.empty(NH, dtype=torch.int32, device=dev),
+                   gain=torch.empty(NH, dtype=torch.float64, device=dev),
+                   n_rows=torch.empty(NH, dtype=torch.int64, device=dev),
+                   n_left=torch.empty(NH, dtype=torch.int64, device=dev))
+        self.ctx.gbdtmo_tree_export(self.p, self.state, rec["node_state"], rec["feature"], rec["bin"], rec["gain"],
+                                    rec["n_rows"], rec["n_left"])
+        rec["leaf"] = self.leaf.clone()
+        return rec
+
+    def fit(self, T: Optional[int] = None):
+        for _ in range(T if T is not None else self.params.T):
+            self.step()
+        return self
+
+    # ----------------------------------------------------------------- graphs
+    def capture(self):
+        """Capture one tree (grad .. update_pred) as a CUDA graph; replay with step_graph()."""
+        s = torch.cuda.Stream(self.device)
+        s.wait_stream(torch.cuda.current_stream(self.device))
+        with torch.cuda.stream(s):
+            self._tree()                      # warm-up outside the graph (allocations, attributes)
+        torch.cuda.current_stream(self.device).wait_stream(s)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            self._tree()
+        self._graph = g
+        return g
+
+    def step_graph(self):
+        self._graph.replay()
+        if self.keep_model:
+            self.trees.append(self.export())
+
+
+def train(X, Y, params: Params, device: str = "cuda:0", ctx: Optional[Context] = None, group=None,
+          f_begin: int = 0, m_global: Optional[int] = None):
+    """Public entry point: X float32 [n][m] and Y float32 [n][d] (host or device tensors or numpy
+    arrays).  Copies the inputs to the GPU, bins the features, trains params.T trees, and
+    returns the Booster (predictions in booster.pred, tree records in booster.trees)."""
+    dev = torch.device(device)
+    ctx = ctx or Context(dev.index or 0)
+    Xt = torch.as_tensor(X)
+    Yt = torch.as_tensor(Y)
+    Xd = Xt.to(dev, non_blocking=True).contiguous()
+    Yd = Yt.to(dev, non_blocking=True).contiguous().float()
+    ds = bin_features(ctx, Xd, params.B, f_begin=f_begin, m_global=m_global)
+    del Xd
+    b = Booster(ctx, ds, Yd, params, group=group)
+    b.fit()
+    return b

@@ -1,0 +1,201 @@
+// common.cuh — context, state layout and launch configuration shared by the kernels
+// of libgbdtmo.so (the product path).  Nothing here is shared with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+
+#include <string>
+
+#include "gbdtmo.h"
+
+namespace gbdtmo {
+
+// ------------------------------------------------------------------ context
+
+struct Ctx {
+  int device = 0;
+  cudaStream_t stream = 0;
+  int num_sms = 148;
+  int max_smem_optin = 227 * 1024;
+  int64_t launches = 0;
+  std::string err;
+};
+
+#define GB_CHECK_ARG(cond, msg)                  \
+  do {                                           \
+    if (!(cond)) {                               \
+      ctx->err = std::string(__func__) + ": " + (msg); \
+      return GBDTMO_EINVAL;                      \
+    }                                            \
+  } while (0)
+
+#define GB_CHECK_LAUNCH()                                                        \
+  do {                                                                           \
+    cudaError_t e_ = cudaGetLastError();                                         \
+    if (e_ != cudaSuccess) {                                                     \
+      ctx->err = std::string(__func__) + ": " + cudaGetErrorString(e_);          \
+      return GBDTMO_ECUDA;                                                       \
+    }                                                                            \
+  } while (0)
+
+// ----------------------------------------------------------------- constants
+
+constexpr int kQShift = 30;            // q = rint(g * 2^30 / P), |q| <= 2^30
+constexpr int kChunkMax = 65536;       // rows per histogram work item: lo-limb sums < 2^32
+constexpr int kChunkMin = 512;
+constexpr int kPartTile = 2048;        // positions per partition block
+constexpr int kHistThreads = 1024;     // histogram CTA (1 CTA / SM, ~200 KB smem)
+constexpr int kHistSmemBudget = 210 * 1024;
+constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte bin window)
+
+enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2 };
+
+__host__ __device__ inline int channels(const gbdtmo_problem& p) {
+  return p.loss == GBDTMO_LOSS_SOFTMAX ? 2 * p.d : p.d;
+}
+__host__ __device__ inline int64_t heap_nodes(const gbdtmo_problem& p) { return (int64_t(1) << (p.D + 1)) - 1; }
+__host__ __device__ inline int64_t max_level_nodes(const gbdtmo_problem& p) { return int64_t(1) << (p.D > 0 ? p.D - 1 : 0); }
+__host__ __device__ inline int64_t max_chunks(const gbdtmo_problem& p) {
+  return p.n / kChunkMin + (int64_t(1) << p.D) + 2;
+}
+__host__ __device__ inline int64_t part_tiles(const gbdtmo_problem& p) { return (p.n + kPartTile - 1) / kPartTile; }
+__host__ __device__ inline int64_t rec_words(const gbdtmo_problem& p) { return channels(p) + 4; }
+__host__ __device__ inline int64_t bitmap_offset(const gbdtmo_problem& p) { return max_level_nodes(p) * rec_words(p); }
+
+// Histogram tiling: a work item is (row chunk, feature tile of
+// k features, channel tile of K channels).  Lanes map to (row-in-group, channel) with
+// K channels per row and 32/K rows per warp instruction.
+struct HistCfg {
+  int K;      // channels per tile (4, 8, 16 or 32)
+  int k;      // features per tile
+  int n_ct;   // channel tiles
+  int n_ft;   // feature tiles
+  int smem;   // bytes of dynamic shared memory
+};
+
+__host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
+  HistCfg c;
+  int V = channels(p);
+  c.K = V <= 4 ? 4 : V <= 8 ? 8 : V <= 16 ? 16 : 32;
+  c.n_ct = (V + c.K - 1) / c.K;
+  int per_feature = p.B * (2 * c.K + 1) * 4;
+  int k = kHistSmemBudget / per_feature;
+  if (k > kMaxTileFeatures) k = kMaxTileFeatures;
+  if (k > p.m) k = p.m;
+  if (k < 1) k = 1;
+  c.k = k;
+  c.n_ft = (p.m + k - 1) / k;
+  c.smem = k * per_feature;
+  return c;
+}
+
+// ------------------------------------------------------------- state layout
+
+struct StateLayout {
+  size_t rows0, rows1, nid;
+  size_t node_begin, node_end, node_state, node_mode, node_feat, node_bin, node_gain, node_nleft, node_sum;
+  size_t chunks, misc, scale_max, tile_cnt, lpart;
+  size_t total;
+};
+
+__host__ __device__ inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+__host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
+  StateLayout L;
+  size_t o = 0;
+  const size_t n = (size_t)p.n, NH = (size_t)heap_nodes(p), V = (size_t)channels(p);
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes, 256); return r; };
+  L.rows0 = take(4 * n);
+  L.rows1 = take(4 * n);
+  L.nid = take(4 * n);
+  L.node_begin = take(4 * NH);
+  L.node_end = take(4 * NH);
+  L.node_state = take(4 * NH);
+  L.node_mode = take(4 * NH);
+  L.node_feat = take(4 * NH);
+  L.node_bin = take(4 * NH);
+  L.node_gain = take(8 * NH);
+  L.node_nleft = take(8 * NH);
+  L.node_sum = take(8 * NH * (V + 1));
+  L.chunks = take(16 * (size_t)max_chunks(p));
+  L.misc = take(64);
+  L.scale_max = take(8 * V);
+  L.tile_cnt = take(4 * ((size_t)part_tiles(p) + 1));
+  L.lpart = take(4 * NH);
+  L.total = o;
+  return L;
+}
+
+// misc words
+enum { MISC_CHUNK_COUNT = 0, MISC_WORK_COUNTER = 1, MISC_CHUNK_ROWS = 2 };
+
+struct State {
+  int32_t *rows0, *rows1, *nid;
+  int32_t *node_begin, *node_end, *node_state, *node_mode, *node_feat, *node_bin;
+  double* node_gain;
+  int64_t* node_nleft;
+  int64_t* node_sum;  // [NH][V+1]: V channel sums of q, then the row count
+  int4* chunks;       // (slot, begin, end, unused)
+  int32_t* misc;
+  unsigned long long* scale_max;   // bits of max_i |g_ic| (fp64, non-negative)
+  int32_t* tile_cnt;
+  int32_t* lpart;
+};
+
+__host__ __device__ inline State state_view(const gbdtmo_problem& p, void* base) {
+  StateLayout L = state_layout(p);
+  char* b = (char*)base;
+  State s;
+  s.rows0 = (int32_t*)(b + L.rows0);
+  s.rows1 = (int32_t*)(b + L.rows1);
+  s.nid = (int32_t*)(b + L.nid);
+  s.node_begin = (int32_t*)(b + L.node_begin);
+  s.node_end = (int32_t*)(b + L.node_end);
+  s.node_state = (int32_t*)(b + L.node_state);
+  s.node_mode = (int32_t*)(b + L.node_mode);
+  s.node_feat = (int32_t*)(b + L.node_feat);
+  s.node_bin = (int32_t*)(b + L.node_bin);
+  s.node_gain = (double*)(b + L.node_gain);
+  s.node_nleft = (int64_t*)(b + L.node_nleft);
+  s.node_sum = (int64_t*)(b + L.node_sum);
+  s.chunks = (int4*)(b + L.chunks);
+  s.misc = (int32_t*)(b + L.misc);
+  s.scale_max = (unsigned long long*)(b + L.scale_max);
+  s.tile_cnt = (int32_t*)(b + L.tile_cnt);
+  s.lpart = (int32_t*)(b + L.lpart);
+  return s;
+}
+
+// ------------------------------------------------------------ validation
+
+inline const char* check_problem(const gbdtmo_problem* p) {
+  if (!p) return "problem is NULL";
+  if (p->n < 1 || p->n >= (int64_t(1) << 31)) return "n out of range [1, 2^31)";
+  if (p->m < 1) return "m < 1";
+  if (p->m_global < p->m || p->f_begin < 0 || p->f_begin + p->m > p->m_global) return "bad feature shard";
+  if (p->d < 1 || p->d > 1024) return "d out of range [1, 1024]";
+  if (p->B < 2 || p->B > 256) return "B out of range [2, 256]";
+  if ((int64_t)p->m_global * p->B >= (int64_t(1) << 24)) return "m_global * B must be < 2^24";
+  if (p->D < 1 || p->D > 12) return "D out of range [1, 12]";
+  if (p->loss != GBDTMO_LOSS_MSE && p->loss != GBDTMO_LOSS_SOFTMAX) return "unknown loss";
+  if (p->min_node < 1) return "min_node < 1";
+  if (!(p->lambda >= 0.0)) return "lambda < 0";
+  if (!(p->gamma >= 0.0)) return "gamma < 0";
+  if (p->ld_bins < p->m || p->ld_bins % 8 != 0) return "ld_bins must be >= m and a multiple of 8";
+  return nullptr;
+}
+
+// Histogram work items wanted per level -> chunks per build level (grad.cu).
+int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p);
+
+// Launch helpers: count kernels and check errors.
+#define GB_LAUNCH(kernel, grid, block, smem, ...)                 \
+  do {                                                            \
+    kernel<<<(grid), (block), (smem), ctx->stream>>>(__VA_ARGS__); \
+    ctx->launches++;                                              \
+    GB_CHECK_LAUNCH();                                            \
+  } while (0)
+
+}  // namespace gbdtmo

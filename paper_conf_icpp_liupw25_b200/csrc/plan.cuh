@@ -1,0 +1,92 @@
+// plan.cuh — device-side level planning: the list of histogram work chunks of a level.
+// Runs inside a single CTA (blockDim.x == 256) so no host round trip is needed.
+#pragma once
+#include "common.cuh"
+
+namespace gbdtmo {
+
+constexpr int kPlanThreads = 256;
+
+// Exclusive scan of one int per thread across a 256-thread block; returns the prefix and
+// writes the block total to *total (all threads).
+__device__ inline int block_excl_scan_256(int v, int* total) {
+  __shared__ int warp_sums[kPlanThreads / 32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_sums[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    int s = lane < kPlanThreads / 32 ? warp_sums[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < kPlanThreads / 32) warp_sums[lane] = s;   // inclusive per warp
+  }
+  __syncthreads();
+  int base = w > 0 ? warp_sums[w - 1] : 0;
+  *total = warp_sums[kPlanThreads / 32 - 1];
+  __syncthreads();
+  return base + x - v;
+}
+
+// Write the build chunks of `level` into s.chunks: every node of the level with mode BUILD
+// is cut into pieces of R rows, R = clamp(ceil(build_rows / target_chunks), kChunkMin, kChunkMax).
+__device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s, int level,
+                                         int target_chunks) {
+  const int64_t LN = int64_t(1) << level, first = LN - 1;
+  __shared__ long long sh_rows;
+  __shared__ int sh_R, sh_base;
+  if (threadIdx.x == 0) { sh_rows = 0; sh_base = 0; }
+  __syncthreads();
+  long long my = 0;
+  for (int64_t i = threadIdx.x; i < LN; i += blockDim.x) {
+    int64_t h = first + i;
+    if (s.node_mode[h] == MODE_BUILD) my += s.node_end[h] - s.node_begin[h];
+  }
+  atomicAdd((unsigned long long*)&sh_rows, (unsigned long long)my);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    long long t = target_chunks > 0 ? target_chunks : 1;
+    long long R = (sh_rows + t - 1) / t;
+    if (R < kChunkMin) R = kChunkMin;
+    if (R > kChunkMax) R = kChunkMax;
+    sh_R = (int)R;
+  }
+  __syncthreads();
+  const int R = sh_R;
+  for (int64_t i0 = 0; i0 < LN; i0 += blockDim.x) {
+    int64_t i = i0 + threadIdx.x;
+    int nchunk = 0, b = 0, e = 0;
+    if (i < LN) {
+      int64_t h = first + i;
+      if (s.node_mode[h] == MODE_BUILD) {
+        b = s.node_begin[h]; e = s.node_end[h];
+        nchunk = (e - b + R - 1) / R;
+      }
+    }
+    int total;
+    int off = block_excl_scan_256(nchunk, &total) + sh_base;
+    for (int c = 0; c < nchunk; ++c) {
+      int cb = b + c * R;
+      int ce = cb + R < e ? cb + R : e;
+      s.chunks[off + c] = make_int4((int)i, cb, ce, 0);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) sh_base += total;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    s.misc[MISC_CHUNK_COUNT] = sh_base;
+    s.misc[MISC_WORK_COUNTER] = 0;
+    s.misc[MISC_CHUNK_ROWS] = R;
+  }
+}
+
+}  // namespace gbdtmo

@@ -1,0 +1,285 @@
+"""CUDA path (through the C ABI) vs the CPU oracle on the same seeded inputs.
+
+Tolerances:
+  bins, cuts, counts, tree structure, partitions  bit-exact (ties: oracle gain at the GPU's
+      choice within 1e-6 relative of the oracle's best, R22)
+  histograms   |gpu - oracle| <= 1e-5 * max(|oracle|, sum|g| of the bin)  (exact on dyadic tree-1 inputs)
+  leaf values / predictions after T trees      <= 1e-4 absolute (north star)
+"""
+import numpy as np
+import pytest
+import torch
+
+from gen import gen
+from tests.gpu_helpers import compare_trees, node_rows, to_np
+
+pytestmark = pytest.mark.gpu
+
+DEV = "cuda:0"
+
+
+@pytest.fixture(scope="module")
+def pkg():
+    import paper_conf_icpp_liupw25_b200 as pkg
+    pkg.lib()
+    return pkg
+
+
+@pytest.fixture(scope="module")
+def ctx(pkg):
+    return pkg.Context(0)
+
+
+def _params(pkg, w, T=None, D=None):
+    return pkg.Params(loss=w.loss, T=T or w.T, D=D or w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
+                      min_node=w.min_node)
+
+
+def _inputs(w):
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    return X, Y
+
+
+CASES = {
+    "C1": gen.WORKLOADS["C1"],
+    "C2s": gen.WORKLOADS["C2"].scaled(n=20_000, m=64, T=3, D=6),
+    "C3s": gen.WORKLOADS["C3"].scaled(n=100_000, m=24, T=3, D=6),
+    "C4s": gen.WORKLOADS["C4"].scaled(n=20_000, m=20, T=2, D=4),
+    "C5s": gen.WORKLOADS["C5"].scaled(n=50_000, m=70, T=2, D=5),
+}
+
+
+# ---------------------------------------------------------------------------- binning
+
+@pytest.mark.parametrize("case", ["C1", "C2s", "C3s", "C4s"])
+def test_bin_matches_oracle(orc, pkg, ctx, case):
+    w = CASES[case]
+    X = gen.features_host(w)
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    torch.cuda.synchronize()
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+    np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+    gb = ds.bins[: w.n * ds.ld_bins].view(w.n, ds.ld_bins)[:, : w.m].cpu().numpy()
+    np.testing.assert_array_equal(gb.T, bins)
+
+
+def test_bin_edge_cases(orc, pkg, ctx):
+    rng = np.random.default_rng(0)
+    n = 9000
+    X = np.stack([
+        np.zeros(n), np.full(n, -3.5), rng.integers(0, 3, n), rng.normal(size=n),
+        np.where(rng.random(n) < 0.5, -0.0, 0.0), rng.integers(0, 300, n),
+        np.concatenate([np.zeros(n - 5), rng.normal(size=5)]), np.arange(n)[::-1],
+    ], axis=1).astype(np.float32)
+    for B in (2, 16, 256):
+        ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), B)
+        torch.cuda.synchronize()
+        cuts, nbins, bins = orc.bin_matrix(X, B)
+        np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+        np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+        gb = ds.bins[: n * ds.ld_bins].view(n, ds.ld_bins)[:, : X.shape[1]].cpu().numpy()
+        np.testing.assert_array_equal(gb.T, bins)
+
+
+# ------------------------------------------------------------------------- gradients
+
+@pytest.mark.parametrize("case", ["C1", "C2s"])
+def test_grad_matches_oracle(orc, pkg, ctx, case):
+    w = CASES[case]
+    X, Y = _inputs(w)
+    rng = np.random.default_rng(1)
+    pred = rng.normal(scale=0.3, size=Y.shape)
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), pred=torch.from_numpy(pred).to(DEV))
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+    ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
+    torch.cuda.synchronize()
+    q = b.q.cpu().numpy().astype(np.float64)
+    sc = b.scales.cpu().numpy().astype(np.float64)
+    assert np.all(np.log2(sc) == np.round(np.log2(sc)))           # powers of two
+    g, h = orc.grad(w.loss, Y.astype(np.float64), pred)
+    d = w.d
+    gq = q[:, :d] * sc[:d]
+    # fp32 arithmetic (2^-23 relative) + fixed-point quantisation (2^-31 P)
+    # fp64 arithmetic (~1e-15) + fixed-point quantisation (half a unit of 2^-30 P)
+    tol = 1e-14 * np.maximum(np.abs(g), 1.0) + sc[:d] * 0.5
+    assert np.all(np.abs(gq - g) <= tol)
+    if w.loss == 1:
+        hq = q[:, d:] * sc[d:]
+        assert np.all(np.abs(hq - h) <= 1e-14 + sc[d:] * 0.5)
+    assert np.all(np.abs(q) <= 2 ** 30)
+
+
+# ------------------------------------------------------------------------ histograms
+
+@pytest.mark.parametrize("case", ["C1", "C3s", "C5s", "C2s", "C4s"])
+def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
+    """Every level's histograms (built and derived by subtraction) vs the oracle's direct
+    per-node histograms over the oracle's node rows; exact on tree-1 dyadic MSE inputs."""
+    w = CASES[case]
+    X, Y = _inputs(w)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=1, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    rows = node_rows(bins, ref["state"][0], ref["feat"][0], ref["bin"][0], w.n)
+    g, h = orc.grad(w.loss, Y.astype(np.float64), np.zeros(Y.shape))
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1))
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+    ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
+    sc = None
+    V, B, m, d = b.p.V, w.B, w.m, w.d
+    checked = 0
+    for lvl in range(w.D):
+        b._level(lvl)
+        torch.cuda.synchronize()
+        if sc is None:
+            sc = b.scales.cpu().numpy().astype(np.float64)
+        if lvl == w.D - 1 and lvl > 0:
+            continue      # derived histograms of the last level are never materialised
+        LN = 1 << lvl
+        H = b.hist[lvl % 2][: LN * m * B * V].view(LN, m, B, V).cpu().numpy()
+        CN = b.cnt[lvl % 2][: LN * m * B].view(LN, m, B).cpu().numpy()
+        for slot in range(LN):
+            hid = LN - 1 + slot
+            if ref["state"][0][hid] != 1:         # only nodes that were searched and split
+                continue
+            r = rows[hid]
+            HG, HH, CNT = orc.build_hist(bins, B, g, h, r)
+            np.testing.assert_array_equal(CN[slot], CNT)
+            gpu_g = H[slot][:, :, :d] * sc[:d]
+            AG = np.zeros((m, B, d))
+            np.add.at(AG, (np.arange(m)[:, None], bins[:, r]), np.abs(g[r])[None, :, :].repeat(m, 0))
+            err = np.abs(gpu_g - HG) / np.maximum(np.maximum(np.abs(HG), AG), 1e-300)
+            assert err.max() <= 1e-5, (lvl, slot, err.max())
+            if w.loss == 0 and w.index in (1, 3, 5):
+                assert np.array_equal(gpu_g, HG), (lvl, slot)      # dyadic tree 1: bit-exact
+            if w.loss == 1:
+                gpu_h = H[slot][:, :, d:] * sc[d:]
+                assert np.all(np.abs(gpu_h - HH) <= 1e-5 * HH + CNT[:, :, None] * 2.0 ** -32)
+            checked += 1
+    assert checked > 0
+
+
+# ------------------------------------------------------------------- whole trees
+
+@pytest.mark.parametrize("case", ["C1", "C2s", "C3s", "C4s", "C5s"])
+def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case):
+    w = CASES[case]
+    X, Y = _inputs(w)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w))
+    b.fit()
+    torch.cuda.synchronize()
+    for t in range(w.T):
+        gt = to_np(b.trees[t])
+        diffs = compare_trees(gt, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t])
+        assert not diffs, (t, diffs)
+        leaves = gt["node_state"] == 2
+        np.testing.assert_allclose(gt["leaf"][leaves], ref["leaf"][t][leaves], rtol=1e-5, atol=1e-6)
+        split = gt["node_state"] == 1
+        np.testing.assert_allclose(gt["gain"][split], ref["gain"][t][split], rtol=1e-6)
+    err = np.max(np.abs(b.pred.cpu().numpy() - ref["pred"]))
+    assert err <= 1e-4, err
+
+
+def test_partition_rows_are_stable_and_complete(orc, pkg, ctx):
+    """After each level the row list of every node equals the oracle's stable partition."""
+    w = CASES["C3s"]
+    X, Y = _inputs(w)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=1, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    rows = node_rows(bins, ref["state"][0], ref["feat"][0], ref["bin"][0], w.n)
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1))
+    b.step()
+    torch.cuda.synchronize()
+    NH = b.NH
+    rl_t = torch.empty(w.n, dtype=torch.int32, device=DEV)
+    nid_t = torch.empty(w.n, dtype=torch.int32, device=DEV)
+    beg_t = torch.empty(NH, dtype=torch.int32, device=DEV)
+    end_t = torch.empty(NH, dtype=torch.int32, device=DEV)
+    ctx.gbdtmo_rows_export(b.p, b.state, w.D, rl_t, nid_t, beg_t, end_t)
+    torch.cuda.synchronize()
+    rl, nid, begin, end = (x.cpu().numpy() for x in (rl_t, nid_t, beg_t, end_t))
+    for hid, r in rows.items():
+        if ref["state"][0][hid] == 2:
+            np.testing.assert_array_equal(rl[begin[hid]:end[hid]], r)
+            assert np.all(nid[r] == hid)
+
+
+def test_two_shards_equal_one(orc, pkg, ctx):
+    """Feature partitioning emulated on one GPU: two shards exchange through
+    MAX(keys) and SUM(xchg) exactly as the NCCL path does; trees and predictions must equal the
+    single-shard run bit for bit."""
+    w = CASES["C3s"]
+    X, Y = _inputs(w)
+    Yd = torch.from_numpy(Y).to(DEV)
+    P = _params(pkg, w, T=2)
+    full = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), Yd.clone(), P)
+    full.fit()
+    half = w.m // 2 + 3
+    shards = []
+    for f0, f1 in ((0, half), (half, w.m)):
+        ds = pkg.bin_features(ctx, torch.from_numpy(np.ascontiguousarray(X[:, f0:f1])).to(DEV), w.B,
+                              f_begin=f0, m_global=w.m)
+        shards.append(pkg.Booster(ctx, ds, Yd.clone(), P))
+    for t in range(P.T):
+        for s in shards:
+            ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+            ctx.gbdtmo_grad(s.p, s.y, s.pred, s.q, s.scales, s.state)
+        for lvl in range(P.D):
+            cur, par = lvl % 2, (lvl - 1) % 2
+            for s in shards:
+                ph = s.hist[par] if lvl else None
+                pc = s.cnt[par] if lvl else None
+                ctx.gbdtmo_build_hist(s.p, lvl, s.ds.bins, s.q, s.state, s.hist[cur], s.cnt[cur])
+                ctx.gbdtmo_find_split(s.p, lvl, s.ds.nbins, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
+                                      s.keys)
+            kmax = torch.maximum(shards[0].keys, shards[1].keys)
+            for s in shards:
+                s.keys.copy_(kmax)
+                ph = s.hist[par] if lvl else None
+                pc = s.cnt[par] if lvl else None
+                ctx.gbdtmo_split_record(s.p, lvl, s.ds.bins, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
+                                        s.keys, s.xchg)
+            xs = shards[0].xchg + shards[1].xchg
+            for s in shards:
+                s.xchg.copy_(xs)
+                ctx.gbdtmo_partition(s.p, lvl, s.state, s.xchg)
+        for s in shards:
+            ctx.gbdtmo_leaf_values(s.p, s.scales, s.state, s.leaf)
+            ctx.gbdtmo_update_pred(s.p, s.state, s.leaf, s.pred)
+            s.trees.append(s.export())
+    torch.cuda.synchronize()
+    for t in range(P.T):
+        a = to_np(full.trees[t])
+        for s in shards:
+            bb = to_np(s.trees[t])
+            for k in ("node_state", "feature", "bin", "n_rows", "n_left"):
+                np.testing.assert_array_equal(a[k], bb[k])
+            np.testing.assert_array_equal(a["leaf"], bb["leaf"])
+    for s in shards:
+        assert torch.equal(full.pred, s.pred)
+
+
+def test_graph_replay_equals_eager(pkg, ctx):
+    w = CASES["C1"]
+    X, Y = _inputs(w)
+    P = _params(pkg, w, T=3)
+    a = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), torch.from_numpy(Y).to(DEV), P)
+    a.fit()
+    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), torch.from_numpy(Y).to(DEV), P)
+    b.capture()          # captures (and its warm-up runs) one tree
+    b.pred.zero_()
+    b.trees.clear()
+    for _ in range(3):
+        b.step_graph()
+    torch.cuda.synchronize()
+    assert torch.equal(a.pred, b.pred)

@@ -81,10 +81,12 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   c.K = V <= 4 ? 4 : V <= 8 ? 8 : V <= 16 ? 16 : 32;
   c.n_ct = (V + c.K - 1) / c.K;
   int per_feature = p.B * (2 * c.K + 1) * 4;
-  int k = kHistSmemBudget / per_feature;
-  if (k > kMaxTileFeatures) k = kMaxTileFeatures;
-  if (k > p.m) k = p.m;
-  if (k < 1) k = 1;
+  int kmax = kHistSmemBudget / per_feature;
+  if (kmax > p.m) kmax = p.m;
+  // compile-time tile widths the kernel is instantiated for
+  const int allowed[9] = {24, 16, 12, 8, 6, 4, 3, 2, 1};
+  int k = 1;
+  for (int i = 0; i < 9; ++i) if (allowed[i] <= kmax) { k = allowed[i]; break; }
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
   c.smem = k * per_feature;

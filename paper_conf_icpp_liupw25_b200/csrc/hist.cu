@@ -19,28 +19,73 @@
 
 namespace gbdtmo {
 
-__device__ __forceinline__ int byte_at(uint64_t w0, uint64_t w1, uint64_t w2, uint64_t w3, int idx) {
-  uint64_t w = (idx < 8) ? w0 : (idx < 16) ? w1 : (idx < 24) ? w2 : w3;
-  return (int)((w >> ((idx & 7) * 8)) & 0xFFu);
+// Raw window of a row's bins: NW 8-byte words starting at the 8-aligned byte f0 & ~7.
+template <int NW>
+struct BinWin { uint64_t w[NW]; };
+
+template <int KF>
+struct HistRow {
+  static constexpr int NW = (KF + 14) / 8;    // raw words: covers (f0 & 7) + KF <= 7 + KF bytes
+  static constexpr int SW = (KF + 7) / 8;     // words after shifting byte (f0 & 7) to position 0
+};
+
+// Shift the raw window right by 8*o bits (o = f0 & 7): byte j of the result = bin of feature f0 + j.
+template <int NW, int SW>
+__device__ __forceinline__ void shift_window(const uint64_t (&w)[NW], int o, uint64_t (&sw)[SW]) {
+  const int sh = 8 * o;
+#pragma unroll
+  for (int i = 0; i < SW; ++i) {
+    const uint64_t lo = w[i] >> sh;
+    const uint64_t hi = (i + 1 < NW && sh) ? (w[i + 1] << (64 - sh)) : 0ull;
+    sw[i] = lo | hi;
+  }
 }
 
-template <int K>
+template <int SW>
+__device__ __forceinline__ uint32_t byte_of(const uint64_t (&sw)[SW], int j) {   // j compile-time after unroll
+  const uint64_t x = sw[j >> 3];
+  const uint32_t half = ((j & 7) < 4) ? (uint32_t)x : (uint32_t)(x >> 32);
+  return __byte_perm(half, 0u, 0x4440u | (uint32_t)(j & 3));                     // PRMT: one byte, zero-extended
+}
+
+// Shared-memory atomic add without return (SASS ATOMS.ADD) at a 32-bit shared address.
+__device__ __forceinline__ void red_shared_add(uint32_t addr, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+
+template <int SW>
+__device__ __forceinline__ int byte_of_rt(const uint64_t (&sw)[SW], int j) {  // j runtime (per lane)
+  uint64_t x = sw[0];
+#pragma unroll
+  for (int i = 1; i < SW; ++i) x = (j >= 8 * i) ? sw[i] : x;
+  return (int)((x >> ((j & 7) * 8)) & 0xFFu);
+}
+
+// K channels per lane group, KF features per tile (both compile-time).
+// Shared layout, bin-major: limbs[b][j][2K] (two halves of K words: the lo and hi limbs),
+// counts[b][KF].  Even rows of a warp instruction put lo in half 0 and hi in half 1, odd rows
+// the other way round, so one instruction's 32 lanes always hit 32 distinct banks.
+template <int K, int KF>
 __global__ void __launch_bounds__(kHistThreads, 1)
 k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ q,
             const int32_t* __restrict__ rows, int use_rows, State s,
             int64_t* __restrict__ hist, int32_t* __restrict__ cnt) {
   extern __shared__ __align__(16) uint32_t sm[];
   __shared__ int sh_item;
-  constexpr int RPI = 32 / K;                 // rows per warp instruction
+  constexpr int RPI = 32 / K;                  // rows per warp instruction
+  constexpr int RS = KF * 2 * K;               // limb words per bin
+  constexpr int NW = HistRow<KF>::NW, SW = HistRow<KF>::SW;
   const int V = channels(p), B = p.B, m = p.m;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
   const int ri = lane / K, c = lane % K;
   const int tiles = hc.n_ft * hc.n_ct;
   const int nitems = s.misc[MISC_CHUNK_COUNT] * tiles;
-  const int limb_words = hc.k * B * 2 * K;
-  uint32_t* limbs = sm;
+  const int limb_words = B * RS;
   uint32_t* cnts = sm + limb_words;
-  const int oa = (ri & 1) ? K : 0, ob = K - oa;   // alternate rows swap limb halves (banks)
+  const int slotA = c + ((ri & 1) ? K : 0), slotB = slotA ^ K;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
+  const uint32_t aA = sbase + 4u * slotA, aB = sbase + 4u * slotB;
+  const int64_t ld = p.ld_bins;
 
   for (;;) {
     if (threadIdx.x == 0) sh_item = atomicAdd(&s.misc[MISC_WORK_COUNTER], 1);
@@ -50,13 +95,12 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int chunk = item / tiles, tile = item - chunk * tiles;
     const int ft = tile / hc.n_ct, ct = tile - ft * hc.n_ct;
     const int4 ch = s.chunks[chunk];
-    const int f0 = ft * hc.k;
-    const int kk = min(hc.k, m - f0);
+    const int f0 = ft * KF;
+    const int kk = min(KF, m - f0);
     const int c0 = ct * K;
     const bool do_cnt = (ct == 0);
 
-    // zero the tile's accumulators
-    const int words = limb_words + hc.k * B;
+    const int words = limb_words + B * KF;
     for (int i = threadIdx.x * 4; i < limb_words; i += blockDim.x * 4)
       *reinterpret_cast<uint4*>(&sm[i]) = make_uint4(0, 0, 0, 0);
     for (int i = limb_words + threadIdx.x; i < words; i += blockDim.x) sm[i] = 0;
@@ -64,37 +108,73 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 
     const int beg = ch.y, end = ch.z;
     const int o = f0 & 7;
-    const int nwin = (o + kk + 7) >> 3;
     const uint8_t* bbase = bins + (f0 & ~7);
     const bool chan_on = (c0 + c) < V;
-    for (int g = beg + warp * RPI; g < end; g += nwarps * RPI) {
-      const int pos = g + ri;
-      if (pos < end) {
-        const int r = use_rows ? __ldg(&rows[pos]) : pos;
-        const int qv = chan_on ? __ldg(&q[(int64_t)r * V + c0 + c]) : 0;
-        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r * p.ld_bins);
-        uint64_t w0 = __ldg(wp), w1 = 0, w2 = 0, w3 = 0;
-        if (nwin > 1) w1 = __ldg(wp + 1);
-        if (nwin > 2) w2 = __ldg(wp + 2);
-        if (nwin > 3) w3 = __ldg(wp + 3);
-        const uint32_t lo = (uint32_t)qv & 0xFFFFu;
-        const uint32_t hi = (uint32_t)(qv >> 16);          // arithmetic shift, two's complement
+    const int step = nwarps * RPI;
+    // software pipeline: row ids two groups ahead, (q, bins) one group ahead
+    int g = beg + warp * RPI;
+    int pos0 = g + ri, pos1 = g + step + ri;
+    int r0 = (pos0 < end) ? (use_rows ? __ldg(&rows[pos0]) : pos0) : -1;
+    int r1 = (pos1 < end) ? (use_rows ? __ldg(&rows[pos1]) : pos1) : -1;
+    int q0 = 0;
+    uint64_t w0[NW];
+#pragma unroll
+    for (int i = 0; i < NW; ++i) w0[i] = 0;
+    if (r0 >= 0) {
+      q0 = chan_on ? __ldg(&q[(int64_t)r0 * V + c0 + c]) : 0;
+      const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r0 * ld);
+#pragma unroll
+      for (int i = 0; i < NW; ++i) w0[i] = __ldg(wp + i);
+    }
+    for (; g < end; g += step) {
+      // issue the loads of the next group and the row id of the one after
+      const int pos2 = g + 2 * step + ri;
+      const int r2 = (pos2 < end) ? (use_rows ? __ldg(&rows[pos2]) : pos2) : -1;
+      int q1 = 0;
+      uint64_t w1[NW];
+#pragma unroll
+      for (int i = 0; i < NW; ++i) w1[i] = 0;
+      if (r1 >= 0) {
+        q1 = chan_on ? __ldg(&q[(int64_t)r1 * V + c0 + c]) : 0;
+        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r1 * ld);
+#pragma unroll
+        for (int i = 0; i < NW; ++i) w1[i] = __ldg(wp + i);
+      }
+      // accumulate the current group
+      if (r0 >= 0) {
+        uint64_t sw[SW];
+        shift_window<NW, SW>(w0, o, sw);
+        const uint32_t lo = (uint32_t)q0 & 0xFFFFu;
+        const uint32_t hi = (uint32_t)(q0 >> 16);          // arithmetic shift, two's complement
         const uint32_t va = (ri & 1) ? hi : lo, vb = (ri & 1) ? lo : hi;
-        uint32_t* lb = limbs + c;
-#pragma unroll 4
-        for (int j = 0; j < kk; ++j) {
-          const int bin = byte_at(w0, w1, w2, w3, o + j);
-          uint32_t* a = lb + (j * B + bin) * (2 * K);
-          atomicAdd(a + oa, va);
-          atomicAdd(a + ob, vb);
+        if (kk == KF) {
+#pragma unroll
+          for (int j = 0; j < KF; ++j) {
+            const uint32_t bin = byte_of<SW>(sw, j);
+            red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+            red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < KF; ++j) {
+            if (j < kk) {
+              const uint32_t bin = byte_of<SW>(sw, j);
+              red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+              red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+            }
+          }
         }
         if (do_cnt) {
-          for (int j = c; j < kk; j += K) {
-            const int bin = byte_at(w0, w1, w2, w3, o + j);
-            atomicAdd(&cnts[j * B + bin], 1u);
+#pragma unroll
+          for (int t = 0; t < (KF + K - 1) / K; ++t) {
+            const int j = c + t * K;
+            if (j < kk) red_shared_add(sbase + 4u * (limb_words + byte_of_rt<SW>(sw, j) * KF + j), 1u);
           }
         }
       }
+      r0 = r1; r1 = r2; q0 = q1;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) w0[i] = w1[i];
     }
     __syncthreads();
 
@@ -105,14 +185,17 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     for (int e = threadIdx.x; e < total; e += blockDim.x) {
       const int cc = e % K, jb = e / K;                        // jb = j * B + b
       if (c0 + cc >= V) continue;
-      const uint32_t los = limbs[jb * 2 * K + cc], his = limbs[jb * 2 * K + K + cc];
+      const int j = jb / B, b = jb - j * B;
+      const uint32_t* rowp = sm + b * RS + j * 2 * K;
+      const uint32_t los = rowp[cc], his = rowp[K + cc];
       const long long v = (long long)(int32_t)his * 65536LL + (long long)los;
       if (v != 0)
         atomicAdd(reinterpret_cast<unsigned long long*>(&hist[(gbase + jb) * V + c0 + cc]), (unsigned long long)v);
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
-        const uint32_t nv = cnts[e];
+        const int j = e / B, b = e - j * B;
+        const uint32_t nv = cnts[b * KF + j];
         if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }
     }
@@ -140,17 +223,34 @@ __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __re
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += stride) cb[i] = 0;
 }
 
+template <int K, int KF>
+static gbdtmo_status launch_hist_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
+                                    const int32_t* q, const int32_t* rows, int use_rows, const State& s,
+                                    int64_t* hist, int32_t* cnt) {
+  static bool attr_done = false;
+  if (!attr_done) {
+    cudaFuncSetAttribute(k_hist_smem<K, KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmemBudget + 4096);
+    attr_done = true;
+  }
+  GB_LAUNCH((k_hist_smem<K, KF>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+  return GBDTMO_OK;
+}
+
 template <int K>
 static gbdtmo_status launch_hist(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
                                  const int32_t* q, const int32_t* rows, int use_rows, const State& s,
                                  int64_t* hist, int32_t* cnt) {
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_smem<K>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmemBudget + 4096);
-    attr_done = true;
+  switch (hc.k) {
+    case 24: return launch_hist_kf<K, 24>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 16: return launch_hist_kf<K, 16>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 12: return launch_hist_kf<K, 12>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 8: return launch_hist_kf<K, 8>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 6: return launch_hist_kf<K, 6>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 4: return launch_hist_kf<K, 4>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 3: return launch_hist_kf<K, 3>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 2: return launch_hist_kf<K, 2>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    default: return launch_hist_kf<K, 1>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
   }
-  GB_LAUNCH(k_hist_smem<K>, ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-  return GBDTMO_OK;
 }
 
 }  // namespace gbdtmo

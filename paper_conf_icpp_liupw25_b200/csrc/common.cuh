@@ -47,7 +47,8 @@ constexpr int kChunkMax = 65536;       // rows per histogram work item: lo-limb 
 constexpr int kChunkMin = 512;
 constexpr int kPartTile = 2048;        // positions per partition block
 constexpr int kHistThreads = 1024;     // histogram CTA (1 CTA / SM, ~200 KB smem)
-constexpr int kHistSmemBudget = 210 * 1024;
+constexpr int kHistSmemBudget = 218 * 1024;   // limbs + counts + per-warp row scratch
+constexpr int kHistWarps = kHistThreads / 32;
 constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte bin window)
 
 enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2 };
@@ -81,15 +82,18 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   c.K = V <= 4 ? 4 : V <= 8 ? 8 : V <= 16 ? 16 : 32;
   c.n_ct = (V + c.K - 1) / c.K;
   int per_feature = p.B * (2 * c.K + 1) * 4;
-  int kmax = kHistSmemBudget / per_feature;
-  if (kmax > p.m) kmax = p.m;
-  // compile-time tile widths the kernel is instantiated for
+  // compile-time tile widths the kernel is instantiated for; each needs a per-warp scratch of
+  // 32 rows x ceil(k/8) 8-byte bin words
   const int allowed[9] = {24, 16, 12, 8, 6, 4, 3, 2, 1};
   int k = 1;
-  for (int i = 0; i < 9; ++i) if (allowed[i] <= kmax) { k = allowed[i]; break; }
+  for (int i = 0; i < 9; ++i) {
+    const int kk = allowed[i];
+    const int need = kk * per_feature + kHistWarps * 32 * 8 * ((kk + 7) / 8);
+    if (kk <= p.m && need <= kHistSmemBudget) { k = kk; break; }
+  }
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
-  c.smem = k * per_feature;
+  c.smem = k * per_feature + kHistWarps * 32 * 8 * ((k + 7) / 8);
   return c;
 }
 

@@ -63,8 +63,14 @@ __device__ __forceinline__ int byte_of_rt(const uint64_t (&sw)[SW], int j) {  //
 
 // K channels per lane group, KF features per tile (both compile-time).
 // Shared layout, bin-major: limbs[b][j][2K] (two halves of K words: the lo and hi limbs),
-// counts[b][KF].  Even rows of a warp instruction put lo in half 0 and hi in half 1, odd rows
-// the other way round, so one instruction's 32 lanes always hit 32 distinct banks.
+// counts[b][KF], then a per-warp scratch of 32 rows x SW bin words.  Even rows of a warp
+// instruction put lo in half 0 and hi in half 1, odd rows the other way round, so one
+// instruction's 32 lanes always hit 32 distinct banks.
+//
+// A warp consumes its rows in batches of 32: lane l loads row l's id and bin window once,
+// shifts it, counts it (CNT) and parks the bins in the scratch; then the K groups of
+// 32/K rows are accumulated, lanes (row, channel) reading their bins back with one LDS and
+// their q value from a batch-wide prefetch.
 template <int K, int KF>
 __global__ void __launch_bounds__(kHistThreads, 1)
 k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ q,
@@ -73,6 +79,8 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   extern __shared__ __align__(16) uint32_t sm[];
   __shared__ int sh_item;
   constexpr int RPI = 32 / K;                  // rows per warp instruction
+  constexpr int G = K;                         // groups per 32-row batch
+  constexpr int SB = G < 8 ? G : 8;            // groups per q-prefetch sub-batch
   constexpr int RS = KF * 2 * K;               // limb words per bin
   constexpr int NW = HistRow<KF>::NW, SW = HistRow<KF>::SW;
   const int V = channels(p), B = p.B, m = p.m;
@@ -81,10 +89,13 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   const int tiles = hc.n_ft * hc.n_ct;
   const int nitems = s.misc[MISC_CHUNK_COUNT] * tiles;
   const int limb_words = B * RS;
-  uint32_t* cnts = sm + limb_words;
+  const int cnt_words = B * KF;
+  uint64_t* scratch = reinterpret_cast<uint64_t*>(sm + limb_words + cnt_words + ((limb_words + cnt_words) & 1)) +
+                      (size_t)warp * 32 * SW;
   const int slotA = c + ((ri & 1) ? K : 0), slotB = slotA ^ K;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sm);
   const uint32_t aA = sbase + 4u * slotA, aB = sbase + 4u * slotB;
+  const uint32_t acnt = sbase + 4u * limb_words;
   const int64_t ld = p.ld_bins;
 
   for (;;) {
@@ -100,7 +111,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int c0 = ct * K;
     const bool do_cnt = (ct == 0);
 
-    const int words = limb_words + B * KF;
+    const int words = limb_words + cnt_words;
     for (int i = threadIdx.x * 4; i < limb_words; i += blockDim.x * 4)
       *reinterpret_cast<uint4*>(&sm[i]) = make_uint4(0, 0, 0, 0);
     for (int i = limb_words + threadIdx.x; i < words; i += blockDim.x) sm[i] = 0;
@@ -110,71 +121,71 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int o = f0 & 7;
     const uint8_t* bbase = bins + (f0 & ~7);
     const bool chan_on = (c0 + c) < V;
-    const int step = nwarps * RPI;
-    // software pipeline: row ids two groups ahead, (q, bins) one group ahead
-    int g = beg + warp * RPI;
-    int pos0 = g + ri, pos1 = g + step + ri;
-    int r0 = (pos0 < end) ? (use_rows ? __ldg(&rows[pos0]) : pos0) : -1;
-    int r1 = (pos1 < end) ? (use_rows ? __ldg(&rows[pos1]) : pos1) : -1;
-    int q0 = 0;
-    uint64_t w0[NW];
+    const int32_t* qc = q + c0 + c;
+    for (int b0 = beg + warp * 32; b0 < end; b0 += nwarps * 32) {
+      // ---- phase 1: lane l owns row b0 + l
+      const int pos = b0 + lane;
+      const bool on = pos < end;
+      int r = -1;
+      if (on) r = use_rows ? __ldg(&rows[pos]) : pos;
+      uint64_t sw[SW];
 #pragma unroll
-    for (int i = 0; i < NW; ++i) w0[i] = 0;
-    if (r0 >= 0) {
-      q0 = chan_on ? __ldg(&q[(int64_t)r0 * V + c0 + c]) : 0;
-      const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r0 * ld);
+      for (int i = 0; i < SW; ++i) sw[i] = 0;
+      if (on) {
+        uint64_t w[NW];
+        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r * ld);
 #pragma unroll
-      for (int i = 0; i < NW; ++i) w0[i] = __ldg(wp + i);
-    }
-    for (; g < end; g += step) {
-      // issue the loads of the next group and the row id of the one after
-      const int pos2 = g + 2 * step + ri;
-      const int r2 = (pos2 < end) ? (use_rows ? __ldg(&rows[pos2]) : pos2) : -1;
-      int q1 = 0;
-      uint64_t w1[NW];
+        for (int i = 0; i < NW; ++i) w[i] = __ldg(wp + i);
+        shift_window<NW, SW>(w, o, sw);
+        if (do_cnt) {
 #pragma unroll
-      for (int i = 0; i < NW; ++i) w1[i] = 0;
-      if (r1 >= 0) {
-        q1 = chan_on ? __ldg(&q[(int64_t)r1 * V + c0 + c]) : 0;
-        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r1 * ld);
-#pragma unroll
-        for (int i = 0; i < NW; ++i) w1[i] = __ldg(wp + i);
+          for (int j = 0; j < KF; ++j)
+            if (j < kk) red_shared_add(acnt + 4u * (byte_of<SW>(sw, j) * KF + j), 1u);
+        }
       }
-      // accumulate the current group
-      if (r0 >= 0) {
-        uint64_t sw[SW];
-        shift_window<NW, SW>(w0, o, sw);
-        const uint32_t lo = (uint32_t)q0 & 0xFFFFu;
-        const uint32_t hi = (uint32_t)(q0 >> 16);          // arithmetic shift, two's complement
-        const uint32_t va = (ri & 1) ? hi : lo, vb = (ri & 1) ? lo : hi;
-        if (kk == KF) {
 #pragma unroll
-          for (int j = 0; j < KF; ++j) {
-            const uint32_t bin = byte_of<SW>(sw, j);
-            red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-            red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
-          }
-        } else {
+      for (int i = 0; i < SW; ++i) scratch[lane * SW + i] = sw[i];
+      __syncwarp();
+      // ---- phase 2: groups of RPI rows x K channels
 #pragma unroll
-          for (int j = 0; j < KF; ++j) {
-            if (j < kk) {
-              const uint32_t bin = byte_of<SW>(sw, j);
-              red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-              red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+      for (int t0 = 0; t0 < G; t0 += SB) {
+        int qv[SB];
+#pragma unroll
+        for (int t = 0; t < SB; ++t) {
+          const int rr = __shfl_sync(0xffffffffu, r, (t0 + t) * RPI + ri);
+          qv[t] = (rr >= 0 && chan_on) ? __ldg(qc + (int64_t)rr * V) : 0;
+        }
+#pragma unroll
+        for (int t = 0; t < SB; ++t) {
+          const int i = (t0 + t) * RPI + ri;
+          if (b0 + i < end) {
+            uint64_t bw[SW];
+#pragma unroll
+            for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
+            const uint32_t lo = (uint32_t)qv[t] & 0xFFFFu;
+            const uint32_t hi = (uint32_t)(qv[t] >> 16);       // arithmetic shift, two's complement
+            const uint32_t va = (ri & 1) ? hi : lo, vb = (ri & 1) ? lo : hi;
+            if (kk == KF) {
+#pragma unroll
+              for (int j = 0; j < KF; ++j) {
+                const uint32_t bin = byte_of<SW>(bw, j);
+                red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+                red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+              }
+            } else {
+#pragma unroll
+              for (int j = 0; j < KF; ++j) {
+                if (j < kk) {
+                  const uint32_t bin = byte_of<SW>(bw, j);
+                  red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+                  red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+                }
+              }
             }
           }
         }
-        if (do_cnt) {
-#pragma unroll
-          for (int t = 0; t < (KF + K - 1) / K; ++t) {
-            const int j = c + t * K;
-            if (j < kk) red_shared_add(sbase + 4u * (limb_words + byte_of_rt<SW>(sw, j) * KF + j), 1u);
-          }
-        }
       }
-      r0 = r1; r1 = r2; q0 = q1;
-#pragma unroll
-      for (int i = 0; i < NW; ++i) w0[i] = w1[i];
+      __syncwarp();
     }
     __syncthreads();
 
@@ -195,7 +206,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
         const int j = e / B, b = e - j * B;
-        const uint32_t nv = cnts[b * KF + j];
+        const uint32_t nv = sm[limb_words + b * KF + j];
         if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }
     }
@@ -229,7 +240,7 @@ static gbdtmo_status launch_hist_kf(Ctx* ctx, const gbdtmo_problem& p, const His
                                     int64_t* hist, int32_t* cnt) {
   static bool attr_done = false;
   if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_smem<K, KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, kHistSmemBudget + 4096);
+    cudaFuncSetAttribute(k_hist_smem<K, KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin - 1024);
     attr_done = true;
   }
   GB_LAUNCH((k_hist_smem<K, KF>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);

@@ -9,48 +9,51 @@
 
 namespace gbdtmo {
 
-constexpr int kFsWarps = 8;      // warps per (node, feature) block; warps split the outputs
-constexpr int kFsFeatures = 4;   // features per block (looped)
-constexpr int kBinsPerLane = 8;  // 32 lanes x 8 contiguous bins = 256 = max B
+constexpr int kFsFeatures = 2;   // features per block (looped)
+constexpr int kFsChunk = 8;      // channels (outputs) scanned together per pass
 
 __device__ __forceinline__ uint64_t pack_key(double gain, int64_t fb) {
   return ((uint64_t)__double_as_longlong(gain) & ~0xFFFFFFull) | (uint64_t)(0xFFFFFF - fb);
 }
 
-// Warp inclusive scan of int64.
-__device__ __forceinline__ long long warp_incl_scan(long long x) {
-  const int lane = threadIdx.x & 31;
+// Block-wide inclusive scan over bins (thread = bin) of N int64 values per thread; also
+// returns the grand totals.  ws: shared [32][N] scratch.
+template <int N>
+__device__ __forceinline__ void block_scan_bins(long long (&v)[N], long long (&tot)[N], long long* ws) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    long long y = __shfl_up_sync(0xffffffffu, x, o);
-    if (lane >= o) x += y;
-  }
-  return x;
-}
-
-// Load the 8 contiguous bins [8 lane, 8 lane + 8) of one histogram channel (stride V between
-// bins) -- for a derived node as parent - sibling, optionally storing the result.
-__device__ __forceinline__ void load_bins_i64(long long v[kBinsPerLane], const int64_t* __restrict__ cur,
-                                              const int64_t* __restrict__ par, const int64_t* __restrict__ sib,
-                                              bool derive, bool store, int64_t stride, int B) {
-  const int lane = threadIdx.x & 31;
 #pragma unroll
-  for (int i = 0; i < kBinsPerLane; ++i) {
-    const int b = lane * kBinsPerLane + i;
-    long long x = 0;
-    if (b < B) {
-      if (derive) {
-        x = par[b * stride] - sib[b * stride];
-        if (store) const_cast<int64_t*>(cur)[b * stride] = x;
-      } else {
-        x = cur[b * stride];
-      }
+    for (int k = 0; k < N; ++k) {
+      const long long y = __shfl_up_sync(0xffffffffu, v[k], o);
+      if (lane >= o) v[k] += y;
     }
-    v[i] = x;
   }
+  if (lane == 31) {
+#pragma unroll
+    for (int k = 0; k < N; ++k) ws[warp * N + k] = v[k];
+  }
+  __syncthreads();
+#pragma unroll
+  for (int k = 0; k < N; ++k) {
+    long long off = 0, t = 0;
+    for (int w = 0; w < nw; ++w) {
+      const long long x = ws[w * N + k];
+      off += (w < warp) ? x : 0;
+      t += x;
+    }
+    v[k] += off;
+    tot[k] = t;
+  }
+  __syncthreads();
 }
 
-__global__ void __launch_bounds__(kFsWarps * 32)
+// One block per (node slot, kFsFeatures features); thread = bin.  For every channel chunk the
+// bins' values (derived nodes: parent - sibling, written back when needed) are prefix-summed
+// across the block; MSE accumulates sum_k G_L^2 and sum_k G_R^2 (H = 2 C is shared by all
+// outputs, so only two divisions per bin are needed), softmax accumulates the Eq. (3) terms.
+template <bool SOFTMAX>
+__global__ void __launch_bounds__(256)
 k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
              State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt,
              const int64_t* __restrict__ phist, const int32_t* __restrict__ pcnt,
@@ -61,139 +64,108 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const bool store = derive && write_derived;
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
-  const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  constexpr bool softmax = SOFTMAX;
+  constexpr int NS = SOFTMAX ? 2 * kFsChunk : kFsChunk;   // scanned values per bin per pass
+  const int b = threadIdx.x;                     // this thread's bin
+  const bool bon = b < B;
   const int sib = slot ^ 1, par = slot >> 1;
   const double lam = p.lambda;
-
-  __shared__ int sh_cl[256 + 1];                 // inclusive prefix counts per bin
-  __shared__ double sh_g[kFsWarps][256];
-  __shared__ double sh_p[kFsWarps];
+  __shared__ long long ws[32 * 2 * kFsChunk];
+  __shared__ unsigned long long wbest[32];
   uint64_t best = 0;
 
   for (int fi = 0; fi < kFsFeatures; ++fi) {
     const int f = blockIdx.x * kFsFeatures + fi;
     if (f >= m) break;
-    const int64_t row_cur = ((int64_t)slot * m + f) * B;
-    const int64_t row_sib = ((int64_t)sib * m + f) * B;
-    const int64_t row_par = ((int64_t)par * m + f) * B;
-    if (warp == 0) {
-      int cv[kBinsPerLane];
-      int run = 0;
+    const int64_t row_cur = ((int64_t)slot * m + f) * B + b;
+    const int64_t row_sib = ((int64_t)sib * m + f) * B + b;
+    const int64_t row_par = ((int64_t)par * m + f) * B + b;
+    // counts
+    long long cv[1] = {0}, ct[1];
+    if (bon) {
+      if (derive) {
+        const int x = pcnt[row_par] - cnt[row_sib];
+        if (store) cnt[row_cur] = x;
+        cv[0] = x;
+      } else {
+        cv[0] = cnt[row_cur];
+      }
+    }
+    block_scan_bins<1>(cv, ct, ws);
+    const long long cl = cv[0], ctot = ct[0];
+    double accL = 0.0, accR = 0.0, P = 0.0;          // MSE: sums of squares; softmax: Eq. (3) terms
+    const int64_t* hc = hist + row_cur * V;
+    const int64_t* hs = hist + row_sib * V;
+    const int64_t* hp = phist + row_par * V;
+    int64_t* hw = hist + row_cur * V;
+    for (int k0 = 0; k0 < d; k0 += kFsChunk) {
+      long long gv[NS], gt[NS];
 #pragma unroll
-      for (int i = 0; i < kBinsPerLane; ++i) {
-        const int b = lane * kBinsPerLane + i;
-        int x = 0;
-        if (b < B) {
+      for (int u = 0; u < kFsChunk; ++u) {
+        const int k = k0 + u;
+        long long x = 0, y = 0;
+        if (bon && k < d) {
           if (derive) {
-            x = pcnt[row_par + b] - cnt[row_sib + b];
-            if (store) cnt[row_cur + b] = x;
+            x = hp[k] - hs[k];
+            if (store) hw[k] = x;
+            if (softmax) { y = hp[d + k] - hs[d + k]; if (store) hw[d + k] = y; }
           } else {
-            x = cnt[row_cur + b];
+            x = hc[k];
+            if (softmax) y = hc[d + k];
           }
         }
-        run += x;
-        cv[i] = run;
+        gv[u] = x;
+        if (SOFTMAX) gv[(kFsChunk + u) % NS] = y;
       }
-      int tot = run;
+      block_scan_bins<NS>(gv, gt, ws);
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(0xffffffffu, tot, o);
-        if (lane >= o) tot += y;
-      }
-      const int excl = tot - run;
-#pragma unroll
-      for (int i = 0; i < kBinsPerLane; ++i) {
-        const int b = lane * kBinsPerLane + i;
-        if (b < 256) sh_cl[b] = excl + cv[i];
-      }
-      if (lane == 31) sh_cl[256] = tot;
-    }
-    __syncthreads();
-    const long long ctot = sh_cl[256];
-
-    double acc[kBinsPerLane];
-#pragma unroll
-    for (int i = 0; i < kBinsPerLane; ++i) acc[i] = 0.0;
-    double ppart = 0.0;
-    for (int k = warp; k < d; k += kFsWarps) {
-      long long gv[kBinsPerLane], hv[kBinsPerLane];
-      load_bins_i64(gv, hist + row_cur * V + k, phist + row_par * V + k, hist + row_sib * V + k, derive, store, V, B);
-      long long run = 0;
-#pragma unroll
-      for (int i = 0; i < kBinsPerLane; ++i) { run += gv[i]; gv[i] = run; }
-      long long tot = warp_incl_scan(run);
-      const long long excl = tot - run;
-      const long long G = __shfl_sync(0xffffffffu, tot, 31);
-      long long H = 0;
-      if (softmax) {
-        load_bins_i64(hv, hist + row_cur * V + d + k, phist + row_par * V + d + k, hist + row_sib * V + d + k,
-                      derive, store, V, B);
-        long long runh = 0;
-#pragma unroll
-        for (int i = 0; i < kBinsPerLane; ++i) { runh += hv[i]; hv[i] = runh; }
-        long long toth = warp_incl_scan(runh);
-        const long long exh = toth - runh;
-        H = __shfl_sync(0xffffffffu, toth, 31);
-#pragma unroll
-        for (int i = 0; i < kBinsPerLane; ++i) hv[i] += exh;
-      }
-      const double sg = (double)scales[k];
-      const double sh = softmax ? (double)scales[d + k] : 0.0;
-      const double Gd = (double)G * sg;
-      const double Hd = softmax ? (double)H * sh : 2.0 * (double)ctot;
-      ppart += Gd * Gd / (Hd + lam);
-#pragma unroll
-      for (int i = 0; i < kBinsPerLane; ++i) {
-        const int b = lane * kBinsPerLane + i;
-        const long long gl = gv[i] + excl;
-        const long long cl = sh_cl[b < 256 ? b : 255];
-        const double GL = (double)gl * sg, GR = (double)(G - gl) * sg;
-        const double HL = softmax ? (double)hv[i] * sh : 2.0 * (double)cl;
-        const double HR = softmax ? (double)(H - hv[i]) * sh : 2.0 * (double)(ctot - cl);
-        acc[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < kBinsPerLane; ++i) {
-      const int b = lane * kBinsPerLane + i;
-      if (b < 256) sh_g[warp][b] = acc[i];
-    }
-    if (lane == 0) sh_p[warp] = ppart;
-    __syncthreads();
-    if (warp == 0) {
-      double P = 0.0;
-#pragma unroll
-      for (int w = 0; w < kFsWarps; ++w) P += sh_p[w];
-      const int nb = nbins[f];
-      const int fg = p.f_begin + f;
-#pragma unroll
-      for (int i = 0; i < kBinsPerLane; ++i) {
-        const int b = lane * kBinsPerLane + i;
-        if (b <= nb - 2 && b < B) {
-          const long long cl = sh_cl[b];
-          if (cl >= p.min_node && ctot - cl >= p.min_node) {
-            double sgain = 0.0;
-#pragma unroll
-            for (int w = 0; w < kFsWarps; ++w) sgain += sh_g[w][b];
-            const double gain = 0.5 * (sgain - P);
-            if (gain > p.gamma) {
-              const uint64_t key = pack_key(gain, (int64_t)fg * B + b);
-              best = key > best ? key : best;
-            }
+      for (int u = 0; u < kFsChunk; ++u) {
+        const int k = k0 + u;
+        if (k < d) {
+          const double sg = (double)scales[k];
+          const double GL = (double)gv[u] * sg, GR = (double)(gt[u] - gv[u]) * sg, G = (double)gt[u] * sg;
+          if (!softmax) {
+            accL = fma(GL, GL, accL);
+            accR = fma(GR, GR, accR);
+            P = fma(G, G, P);
+          } else {
+            const double sh = (double)scales[d + k];
+            const int uh = (kFsChunk + u) % NS;
+            const double HL = (double)gv[uh] * sh, H = (double)gt[uh] * sh;
+            const double HR = (double)(gt[uh] - gv[uh]) * sh;
+            accL += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+            P += G * G / (H + lam);
           }
         }
       }
     }
-    __syncthreads();
+    if (bon && b <= nbins[f] - 2 && cl >= p.min_node && ctot - cl >= p.min_node) {
+      double gain;
+      if (!softmax) {
+        gain = 0.5 * (accL / (2.0 * (double)cl + lam) + accR / (2.0 * (double)(ctot - cl) + lam) -
+                      P / (2.0 * (double)ctot + lam));
+      } else {
+        gain = 0.5 * (accL - P);
+      }
+      if (gain > p.gamma) {
+        const uint64_t key = pack_key(gain, (int64_t)(p.f_begin + f) * B + b);
+        best = key > best ? key : best;
+      }
+    }
   }
-  if (warp == 0) {
+  // block max of the packed keys -> one atomicMax per block
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
-      best = y > best ? y : best;
-    }
-    if (lane == 0 && best) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)best);
+  for (int o = 16; o > 0; o >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
+    best = y > best ? y : best;
+  }
+  if (lane == 0) wbest[warp] = best;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint64_t bb = 0;
+    for (int w = 0; w < nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
+    if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
   }
 }
 
@@ -319,7 +291,9 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   const int64_t LN = int64_t(1) << level;
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
   dim3 grid((p->m + kFsFeatures - 1) / kFsFeatures, (unsigned)LN);
-  GB_LAUNCH(k_find_split, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt,
+  const int threads = ((p->B + 31) / 32) * 32;
+  auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_find_split<true> : k_find_split<false>;
+  GB_LAUNCH(kern, grid, threads, 0, *p, level, nbins, scales, s, hist, cnt,
             level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
   return GBDTMO_OK;
 }

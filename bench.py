@@ -105,10 +105,6 @@ class ClockSampler:
 
 # ---------------------------------------------------------------------------- setup
 
-def shard_range(m, rank, world):
-    return (m * rank) // world, (m * (rank + 1)) // world
-
-
 def built_rows(tree_np, D):
     """Rows whose histograms were built (root + smaller child of every split with a searched child)."""
     st, nr, nl = tree_np["node_state"], tree_np["n_rows"], tree_np["n_left"]
@@ -207,6 +203,7 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
         group = dist.group.WORLD
+    from paper_conf_icpp_liupw25_b200.parallel import shard_range
     f0, f1 = shard_range(w.m, rank, world)
     m_loc = f1 - f0
     ctx = pkg.Context(local)

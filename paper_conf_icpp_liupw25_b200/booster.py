@@ -16,6 +16,7 @@ from typing import Optional
 import torch
 
 from . import _abi
+from . import parallel
 from ._abi import Context, Problem, LOSS_MSE, LOSS_SOFTMAX
 
 
@@ -126,11 +127,11 @@ class Booster:
         ctx.gbdtmo_find_split(p, lvl, self.ds.nbins, self.scales, self.state, self.hist[cur], self.cnt[cur],
                               ph, pc, self.keys)
         if self.group is not None:
-            torch.distributed.all_reduce(self.keys[: 1 << lvl], op=torch.distributed.ReduceOp.MAX, group=self.group)
+            parallel.exchange_keys(self.keys[: 1 << lvl], self.group)
         ctx.gbdtmo_split_record(p, lvl, self.ds.bins, self.scales, self.state, self.hist[cur], self.cnt[cur],
                                 ph, pc, self.keys, self.xchg)
         if self.group is not None:
-            torch.distributed.all_reduce(self.xchg, op=torch.distributed.ReduceOp.SUM, group=self.group)
+            parallel.exchange_records(self.xchg, self.group)
         ctx.gbdtmo_partition(p, lvl, self.state, self.xchg)
 
     def _tree(self, time_hist: bool = False):

@@ -108,7 +108,8 @@ size_t gbdtmo_bins_bytes(int64_t n, int64_t ld_bins);
 size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B);
 /* Opaque per-tree state (row lists, per-row node ids, heap node tables, launch plans). */
 gbdtmo_status gbdtmo_state_bytes(const gbdtmo_problem* p, size_t* bytes /* host */);
-/* Histogram buffers of one level: hist int64 [2^level][m][B][V], cnt int32 [2^level][m][B]. */
+/* Histogram buffers of one level: hist int64 [2^level][m][V][B] (channel-major: bins contiguous),
+ * cnt int32 [2^level][m][B]. */
 gbdtmo_status gbdtmo_hist_bytes(const gbdtmo_problem* p, int32_t level, size_t* hist_bytes, size_t* cnt_bytes);
 /* Exchange buffer (int64 elements): 2^(D-1) split records of V+4 words, then ceil(n/64) bitmap words. */
 gbdtmo_status gbdtmo_xchg_count(const gbdtmo_problem* p, int64_t* count /* host */);
@@ -147,7 +148,7 @@ gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* 
 
 /* For every node of `level` marked "build" by the plan in `state` (the root at level 0, the
  * smaller child of each split afterwards, reading R19), for every local feature f, bin b and
- * channel c:   hist[slot][f][b][c] = sum_{i in node, bin(i,f) = b} q[i][c]   (exact int64),
+ * channel c:   hist[slot][f][c][b] = sum_{i in node, bin(i,f) = b} q[i][c]   (exact int64),
  *              cnt [slot][f][b]    = #{i in node : bin(i,f) = b}.
  * (§3.3; the paper's Alg. 2 body is missing.)
  * bins uint8 with ld = p->ld_bins and gbdtmo_bins_bytes() of storage; q from gbdtmo_grad;

@@ -1,7 +1,7 @@
 // hist.cu — (a)3: per-node histogram build (§3.3; Alg. 2's body is missing,
 // PAPER.md:216-218, so the kernel is designed for sm_100a from the definition):
 //
-//   hist[slot][f][b][c] = sum_{i in node, bin(i,f) = b} q[i][c],   cnt[slot][f][b] = #{...}
+//   hist[slot][f][c][b] = sum_{i in node, bin(i,f) = b} q[i][c],   cnt[slot][f][b] = #{...}
 //
 // B200 design:
 //  - persistent CTAs (1 per SM, ~200 KB shared memory) pull work items (row chunk x feature
@@ -200,8 +200,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       const uint32_t* rowp = sm + b * RS + j * 2 * K;
       const uint32_t los = rowp[cc], his = rowp[K + cc];
       const long long v = (long long)(int32_t)his * 65536LL + (long long)los;
-      if (v != 0)
-        atomicAdd(reinterpret_cast<unsigned long long*>(&hist[(gbase + jb) * V + c0 + cc]), (unsigned long long)v);
+      if (v != 0)   // channel-major node histogram: [f][c][b]
+        atomicAdd(reinterpret_cast<unsigned long long*>(&hist[((slot * m + f0 + j) * V + c0 + cc) * B + b]),
+                  (unsigned long long)v);
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {

@@ -9,51 +9,70 @@
 
 namespace gbdtmo {
 
-constexpr int kFsFeatures = 2;   // features per block (looped)
-constexpr int kFsChunk = 8;      // channels (outputs) scanned together per pass
+constexpr int kFsWarps = 8;      // warps per block = features of one node per block
+constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 
 __device__ __forceinline__ uint64_t pack_key(double gain, int64_t fb) {
   return ((uint64_t)__double_as_longlong(gain) & ~0xFFFFFFull) | (uint64_t)(0xFFFFFF - fb);
 }
 
-// Block-wide inclusive scan over bins (thread = bin) of N int64 values per thread; also
-// returns the grand totals.  ws: shared [32][N] scratch.
-template <int N>
-__device__ __forceinline__ void block_scan_bins(long long (&v)[N], long long (&tot)[N], long long* ws) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+// Exclusive prefix (over lanes) and total of a per-lane int64.
+__device__ __forceinline__ long long warp_excl(long long x, long long* total) {
+  const int lane = threadIdx.x & 31;
+  long long v = x;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-#pragma unroll
-    for (int k = 0; k < N; ++k) {
-      const long long y = __shfl_up_sync(0xffffffffu, v[k], o);
-      if (lane >= o) v[k] += y;
-    }
+    const long long y = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += y;
   }
-  if (lane == 31) {
-#pragma unroll
-    for (int k = 0; k < N; ++k) ws[warp * N + k] = v[k];
-  }
-  __syncthreads();
-#pragma unroll
-  for (int k = 0; k < N; ++k) {
-    long long off = 0, t = 0;
-    for (int w = 0; w < nw; ++w) {
-      const long long x = ws[w * N + k];
-      off += (w < warp) ? x : 0;
-      t += x;
-    }
-    v[k] += off;
-    tot[k] = t;
-  }
-  __syncthreads();
+  *total = __shfl_sync(0xffffffffu, v, 31);
+  return v - x;
 }
 
-// One block per (node slot, kFsFeatures features); thread = bin.  For every channel chunk the
-// bins' values (derived nodes: parent - sibling, written back when needed) are prefix-summed
-// across the block; MSE accumulates sum_k G_L^2 and sum_k G_R^2 (H = 2 C is shared by all
-// outputs, so only two divisions per bin are needed), softmax accumulates the Eq. (3) terms.
+// 8 consecutive int64 bins [8 lane, 8 lane + 8) of one channel row (bins contiguous), for a
+// derived node parent - sibling (written back when `store`); inclusive in-lane prefix on return.
+__device__ __forceinline__ void load_row8(long long (&v)[kFsBins], const int64_t* cur, const int64_t* par,
+                                          const int64_t* sib, bool derive, bool store, int B) {
+  const int lane = threadIdx.x & 31;
+  const int b0 = lane * kFsBins;
+  if (b0 + kFsBins <= B) {
+    const longlong2* pc = reinterpret_cast<const longlong2*>(cur + b0);
+    if (derive) {
+      const longlong2* pp = reinterpret_cast<const longlong2*>(par + b0);
+      const longlong2* ps = reinterpret_cast<const longlong2*>(sib + b0);
+#pragma unroll
+      for (int i = 0; i < kFsBins / 2; ++i) {
+        const longlong2 a = pp[i], c = ps[i];
+        const longlong2 x = make_longlong2(a.x - c.x, a.y - c.y);
+        if (store) const_cast<longlong2*>(pc)[i] = x;
+        v[2 * i] = x.x; v[2 * i + 1] = x.y;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < kFsBins / 2; ++i) { const longlong2 x = pc[i]; v[2 * i] = x.x; v[2 * i + 1] = x.y; }
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < kFsBins; ++i) {
+      const int b = b0 + i;
+      long long x = 0;
+      if (b < B) {
+        if (derive) { x = par[b] - sib[b]; if (store) const_cast<int64_t*>(cur)[b] = x; }
+        else x = cur[b];
+      }
+      v[i] = x;
+    }
+  }
+#pragma unroll
+  for (int i = 1; i < kFsBins; ++i) v[i] += v[i - 1];
+}
+
+// One warp per (node, feature); lane l owns bins [8l, 8l + 8).  Per channel the warp reads the
+// contiguous row of B int64 bins (channel-major histogram: coalesced 16-byte loads), prefix-sums
+// it (in-lane + warp scan), and accumulates per bin: MSE sum_k G_L^2 and sum_k G_R^2 (H = 2 C is
+// shared by all outputs: two divisions per bin), softmax the Eq. (3) terms.
 template <bool SOFTMAX>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(kFsWarps * 32)
 k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
              State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt,
              const int64_t* __restrict__ phist, const int32_t* __restrict__ pcnt,
@@ -64,97 +83,97 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const bool store = derive && write_derived;
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
-  constexpr bool softmax = SOFTMAX;
-  constexpr int NS = SOFTMAX ? 2 * kFsChunk : kFsChunk;   // scanned values per bin per pass
-  const int b = threadIdx.x;                     // this thread's bin
-  const bool bon = b < B;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int f = blockIdx.x * kFsWarps + warp;
   const int sib = slot ^ 1, par = slot >> 1;
   const double lam = p.lambda;
-  __shared__ long long ws[32 * 2 * kFsChunk];
-  __shared__ unsigned long long wbest[32];
+  __shared__ unsigned long long wbest[kFsWarps];
   uint64_t best = 0;
-
-  for (int fi = 0; fi < kFsFeatures; ++fi) {
-    const int f = blockIdx.x * kFsFeatures + fi;
-    if (f >= m) break;
-    const int64_t row_cur = ((int64_t)slot * m + f) * B + b;
-    const int64_t row_sib = ((int64_t)sib * m + f) * B + b;
-    const int64_t row_par = ((int64_t)par * m + f) * B + b;
+  if (f < m) {
     // counts
-    long long cv[1] = {0}, ct[1];
-    if (bon) {
-      if (derive) {
-        const int x = pcnt[row_par] - cnt[row_sib];
-        if (store) cnt[row_cur] = x;
-        cv[0] = x;
-      } else {
-        cv[0] = cnt[row_cur];
-      }
-    }
-    block_scan_bins<1>(cv, ct, ws);
-    const long long cl = cv[0], ctot = ct[0];
-    double accL = 0.0, accR = 0.0, P = 0.0;          // MSE: sums of squares; softmax: Eq. (3) terms
-    const int64_t* hc = hist + row_cur * V;
-    const int64_t* hs = hist + row_sib * V;
-    const int64_t* hp = phist + row_par * V;
-    int64_t* hw = hist + row_cur * V;
-    for (int k0 = 0; k0 < d; k0 += kFsChunk) {
-      long long gv[NS], gt[NS];
+    long long cl[kFsBins];
+    {
+      const int64_t oc = ((int64_t)slot * m + f) * B, os = ((int64_t)sib * m + f) * B, op = ((int64_t)par * m + f) * B;
+      const int b0 = lane * kFsBins;
 #pragma unroll
-      for (int u = 0; u < kFsChunk; ++u) {
-        const int k = k0 + u;
-        long long x = 0, y = 0;
-        if (bon && k < d) {
-          if (derive) {
-            x = hp[k] - hs[k];
-            if (store) hw[k] = x;
-            if (softmax) { y = hp[d + k] - hs[d + k]; if (store) hw[d + k] = y; }
-          } else {
-            x = hc[k];
-            if (softmax) y = hc[d + k];
+      for (int i = 0; i < kFsBins; ++i) {
+        const int b = b0 + i;
+        long long x = 0;
+        if (b < B) {
+          if (derive) { x = pcnt[op + b] - cnt[os + b]; if (store) cnt[oc + b] = (int32_t)x; }
+          else x = cnt[oc + b];
+        }
+        cl[i] = x;
+      }
+#pragma unroll
+      for (int i = 1; i < kFsBins; ++i) cl[i] += cl[i - 1];
+      long long ctot;
+      const long long ex = warp_excl(cl[kFsBins - 1], &ctot);
+#pragma unroll
+      for (int i = 0; i < kFsBins; ++i) cl[i] += ex;
+      cl[0] = cl[0];  // (keeps the array in registers)
+      // ---- channels
+      const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
+                    rowp = ((int64_t)par * m + f) * V * B;
+      double accL[kFsBins], accR[kFsBins];
+#pragma unroll
+      for (int i = 0; i < kFsBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
+      double P = 0.0;
+      for (int k = 0; k < d; ++k) {
+        long long gv[kFsBins];
+        load_row8(gv, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
+                  derive, store, B);
+        long long G;
+        const long long gex = warp_excl(gv[kFsBins - 1], &G);
+        const double sg = (double)scales[k];
+        if (!SOFTMAX) {
+#pragma unroll
+          for (int i = 0; i < kFsBins; ++i) {
+            const double GL = (double)(gv[i] + gex) * sg, GR = (double)(G - gv[i] - gex) * sg;
+            accL[i] = fma(GL, GL, accL[i]);
+            accR[i] = fma(GR, GR, accR[i]);
+          }
+          const double Gd = (double)G * sg;
+          P = fma(Gd, Gd, P);
+        } else {
+          long long hv[kFsBins];
+          load_row8(hv, hist + rowc + (int64_t)(d + k) * B, phist + rowp + (int64_t)(d + k) * B,
+                    hist + rows_ + (int64_t)(d + k) * B, derive, store, B);
+          long long H;
+          const long long hex = warp_excl(hv[kFsBins - 1], &H);
+          const double sh = (double)scales[d + k];
+#pragma unroll
+          for (int i = 0; i < kFsBins; ++i) {
+            const double GL = (double)(gv[i] + gex) * sg, GR = (double)(G - gv[i] - gex) * sg;
+            const double HL = (double)(hv[i] + hex) * sh, HR = (double)(H - hv[i] - hex) * sh;
+            accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+          }
+          const double Gd = (double)G * sg, Hd = (double)H * sh;
+          P += Gd * Gd / (Hd + lam);
+        }
+      }
+      // ---- gains and the lane's best candidate
+      const int nb = nbins[f];
+      const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
+#pragma unroll
+      for (int i = 0; i < kFsBins; ++i) {
+        const int b = b0 + i;
+        const long long c = cl[i];
+        if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
+          double gain;
+          if (!SOFTMAX)
+            gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
+                          P / (2.0 * (double)ctot + lam));
+          else
+            gain = 0.5 * (accL[i] - P);
+          if (gain > p.gamma) {
+            const uint64_t key = pack_key(gain, fb0 + b);
+            best = key > best ? key : best;
           }
         }
-        gv[u] = x;
-        if (SOFTMAX) gv[(kFsChunk + u) % NS] = y;
-      }
-      block_scan_bins<NS>(gv, gt, ws);
-#pragma unroll
-      for (int u = 0; u < kFsChunk; ++u) {
-        const int k = k0 + u;
-        if (k < d) {
-          const double sg = (double)scales[k];
-          const double GL = (double)gv[u] * sg, GR = (double)(gt[u] - gv[u]) * sg, G = (double)gt[u] * sg;
-          if (!softmax) {
-            accL = fma(GL, GL, accL);
-            accR = fma(GR, GR, accR);
-            P = fma(G, G, P);
-          } else {
-            const double sh = (double)scales[d + k];
-            const int uh = (kFsChunk + u) % NS;
-            const double HL = (double)gv[uh] * sh, H = (double)gt[uh] * sh;
-            const double HR = (double)(gt[uh] - gv[uh]) * sh;
-            accL += GL * GL / (HL + lam) + GR * GR / (HR + lam);
-            P += G * G / (H + lam);
-          }
-        }
-      }
-    }
-    if (bon && b <= nbins[f] - 2 && cl >= p.min_node && ctot - cl >= p.min_node) {
-      double gain;
-      if (!softmax) {
-        gain = 0.5 * (accL / (2.0 * (double)cl + lam) + accR / (2.0 * (double)(ctot - cl) + lam) -
-                      P / (2.0 * (double)ctot + lam));
-      } else {
-        gain = 0.5 * (accL - P);
-      }
-      if (gain > p.gamma) {
-        const uint64_t key = pack_key(gain, (int64_t)(p.f_begin + f) * B + b);
-        best = key > best ? key : best;
       }
     }
   }
-  // block max of the packed keys -> one atomicMax per block
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
@@ -164,7 +183,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   __syncthreads();
   if (threadIdx.x == 0) {
     uint64_t bb = 0;
-    for (int w = 0; w < nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
+    for (int w = 0; w < kFsWarps; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
     if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
   }
 }
@@ -203,11 +222,15 @@ __global__ void k_split_record(gbdtmo_problem p, int level, State s, const int64
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const int sib = slot ^ 1, par = slot >> 1;
   const int64_t rc = ((int64_t)slot * m + fl) * B, rs = ((int64_t)sib * m + fl) * B, rp = ((int64_t)par * m + fl) * B;
-  for (int c = threadIdx.x; c < V; c += blockDim.x) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  for (int c = warp; c < V; c += nw) {          // hist is [slot][f][c][b]: a warp sums bins <= b of channel c
     long long acc = 0;
-    for (int bb = 0; bb <= b; ++bb)
-      acc += derive ? (phist[(rp + bb) * V + c] - hist[(rs + bb) * V + c]) : hist[(rc + bb) * V + c];
-    rec[c] = acc;
+    for (int bb = lane; bb <= b; bb += 32)
+      acc += derive ? (phist[(rp * V) + (int64_t)c * B + bb] - hist[(rs * V) + (int64_t)c * B + bb])
+                    : hist[(rc * V) + (int64_t)c * B + bb];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) rec[c] = acc;
   }
   if (threadIdx.x == 0) {
     long long cl = 0;
@@ -290,10 +313,9 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
-  dim3 grid((p->m + kFsFeatures - 1) / kFsFeatures, (unsigned)LN);
-  const int threads = ((p->B + 31) / 32) * 32;
+  dim3 grid((p->m + kFsWarps - 1) / kFsWarps, (unsigned)LN);
   auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_find_split<true> : k_find_split<false>;
-  GB_LAUNCH(kern, grid, threads, 0, *p, level, nbins, scales, s, hist, cnt,
+  GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt,
             level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
   return GBDTMO_OK;
 }

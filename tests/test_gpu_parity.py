@@ -140,7 +140,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
         if lvl == w.D - 1 and lvl > 0:
             continue      # derived histograms of the last level are never materialised
         LN = 1 << lvl
-        H = b.hist[lvl % 2][: LN * m * B * V].view(LN, m, B, V).cpu().numpy()
+        H = b.hist[lvl % 2][: LN * m * V * B].view(LN, m, V, B).transpose(2, 3).cpu().numpy()
         CN = b.cnt[lvl % 2][: LN * m * B].view(LN, m, B).cpu().numpy()
         for slot in range(LN):
             hid = LN - 1 + slot

@@ -63,7 +63,7 @@ __device__ __forceinline__ int byte_of_rt(const uint64_t (&sw)[SW], int j) {  //
 
 // K channels per lane group, KF features per tile (both compile-time).
 // Shared layout, bin-major: limbs[b][j][2K] (two halves of K words: the lo and hi limbs),
-// counts[b][KF], then a per-warp scratch of 32 rows x SW bin words.  Even rows of a warp
+// counts[KF][b], then a per-warp scratch of 32 rows x SW bin words.  Even rows of a warp
 // instruction put lo in half 0 and hi in half 1, odd rows the other way round, so one
 // instruction's 32 lanes always hit 32 distinct banks.
 //
@@ -140,7 +140,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         if (do_cnt) {
 #pragma unroll
           for (int j = 0; j < KF; ++j)
-            if (j < kk) red_shared_add(acnt + 4u * (byte_of<SW>(sw, j) * KF + j), 1u);
+            if (j < kk) red_shared_add(acnt + 4u * (j * B + byte_of<SW>(sw, j)), 1u);   // counts[j][b]: bank = b mod 32
         }
       }
 #pragma unroll
@@ -207,7 +207,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
         const int j = e / B, b = e - j * B;
-        const uint32_t nv = sm[limb_words + b * KF + j];
+        const uint32_t nv = sm[limb_words + e];                    // counts[j][b], e = j * B + b
         if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }
     }

@@ -46,6 +46,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--graph", action="store_true", help="replay each tree as a CUDA graph (1 GPU)")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N > 1 (gloo: lets N ranks share one GPU for testing)")
     return ap.parse_args()
 
 
@@ -197,11 +199,15 @@ def main():
     import torch.distributed as dist
     import paper_conf_icpp_liupw25_b200 as pkg
 
+    local = local % torch.cuda.device_count()       # (ranks may share a GPU with --backend gloo)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if a.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
         group = dist.group.WORLD
     from paper_conf_icpp_liupw25_b200.parallel import shard_range
     f0, f1 = shard_range(w.m, rank, world)

@@ -1,0 +1,77 @@
+"""The Booster's multi-rank path (feature shards + torch.distributed exchanges)
+run as two processes sharing cuda:0 over a gloo group: trees and predictions must equal the
+single-process run bit for bit.  (NCCL needs one GPU per rank; the exchange code is the same.)"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.multiprocessing as mp
+
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _case():
+    from gen import gen
+    return gen.WORKLOADS["C3"].scaled(n=60_000, m=30, T=2, D=5)
+
+
+def _worker(rank, world, port, out):
+    import sys
+    sys.path.insert(0, ROOT)
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_icpp_liupw25_b200 as pkg
+    from paper_conf_icpp_liupw25_b200.parallel import shard_range
+    from gen import gen
+    w = _case()
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    f0, f1 = shard_range(w.m, rank, world)
+    ctx = pkg.Context(0)
+    ds = pkg.bin_features(ctx, torch.from_numpy(np.ascontiguousarray(X[:, f0:f1])).cuda(), w.B, f_begin=f0,
+                          m_global=w.m)
+    P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).cuda(), P, group=dist.group.WORLD)
+    b.fit()
+    torch.cuda.synchronize()
+    out[rank] = ([{k: v.cpu().numpy() for k, v in t.items()} for t in b.trees], b.pred.cpu().numpy())
+    dist.destroy_process_group()
+
+
+def test_two_rank_booster_equals_single_rank():
+    import sys
+    sys.path.insert(0, ROOT)
+    import paper_conf_icpp_liupw25_b200 as pkg
+    from gen import gen
+    w = _case()
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    ctx = pkg.Context(0)
+    P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+    ref = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P)
+    ref.fit()
+    torch.cuda.synchronize()
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.start_processes(_worker, args=(2, _free_port(), out), nprocs=2, join=True, start_method="spawn")
+    for rank in range(2):
+        trees, pred = out[rank]
+        for t in range(w.T):
+            a = {k: v.cpu().numpy() for k, v in ref.trees[t].items()}
+            for k in ("node_state", "feature", "bin", "n_rows", "n_left", "leaf"):
+                np.testing.assert_array_equal(trees[t][k], a[k])
+        np.testing.assert_array_equal(pred, ref.pred.cpu().numpy())

@@ -122,21 +122,35 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const uint8_t* bbase = bins + (f0 & ~7);
     const bool chan_on = (c0 + c) < V;
     const int32_t* qc = q + c0 + c;
-    for (int b0 = beg + warp * 32; b0 < end; b0 += nwarps * 32) {
+    // cross-batch pipeline: row ids two batches ahead, bin windows one batch ahead
+    const int bstep = nwarps * 32;
+    auto load_rid = [&](int pos) -> int { return pos < end ? (use_rows ? __ldg(&rows[pos]) : pos) : -1; };
+    auto load_win = [&](int rr, uint64_t (&w)[NW]) {
+      if (rr >= 0) {
+        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)rr * ld);
+#pragma unroll
+        for (int i = 0; i < NW; ++i) w[i] = __ldg(wp + i);
+      } else {
+#pragma unroll
+        for (int i = 0; i < NW; ++i) w[i] = 0;
+      }
+    };
+    int r_cur = load_rid(beg + warp * 32 + lane);
+    int r_nxt = load_rid(beg + warp * 32 + bstep + lane);
+    uint64_t w_cur[NW];
+    load_win(r_cur, w_cur);
+    for (int b0 = beg + warp * 32; b0 < end; b0 += bstep) {
+      // ---- prefetch for the next batches
+      const int r_nn = load_rid(b0 + 2 * bstep + lane);
+      uint64_t w_nxt[NW];
+      load_win(r_nxt, w_nxt);
       // ---- phase 1: lane l owns row b0 + l
-      const int pos = b0 + lane;
-      const bool on = pos < end;
-      int r = -1;
-      if (on) r = use_rows ? __ldg(&rows[pos]) : pos;
+      const int r = r_cur;
       uint64_t sw[SW];
 #pragma unroll
       for (int i = 0; i < SW; ++i) sw[i] = 0;
-      if (on) {
-        uint64_t w[NW];
-        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)r * ld);
-#pragma unroll
-        for (int i = 0; i < NW; ++i) w[i] = __ldg(wp + i);
-        shift_window<NW, SW>(w, o, sw);
+      if (r >= 0) {
+        shift_window<NW, SW>(w_cur, o, sw);
         if (do_cnt) {
 #pragma unroll
           for (int j = 0; j < KF; ++j)
@@ -186,6 +200,10 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         }
       }
       __syncwarp();
+      r_cur = r_nxt;
+      r_nxt = r_nn;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) w_cur[i] = w_nxt[i];
     }
     __syncthreads();
 
@@ -290,7 +308,6 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
   switch (hc.K) {
     case 4: return launch_hist<4>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
     case 8: return launch_hist<8>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 16: return launch_hist<16>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    default: return launch_hist<32>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    default: return launch_hist<16>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
   }
 }

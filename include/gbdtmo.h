@@ -131,6 +131,15 @@ gbdtmo_status gbdtmo_bin(gbdtmo_ctx ctx, const float* X, int64_t n, int32_t m, i
                          uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                          void* ws, size_t ws_bytes);
 
+/* Sparsity-aware default bins (zeros are implicit in the paper's CSC
+ * storage; here every feature's most frequent bin plays that role): dflt[f] = the bin of feature
+ * f holding the most of the n rows (ties: smallest bin), or -1 when that bin holds fewer than
+ * min_count rows.  The histogram calls skip rows whose bin is the default and recover that bin
+ * exactly as node total - sum of the other bins.
+ * bins as produced by gbdtmo_bin; dflt int32 [m] (out). */
+gbdtmo_status gbdtmo_default_bins(gbdtmo_ctx ctx, const uint8_t* bins, int64_t n, int32_t m, int64_t ld_bins,
+                                  int32_t B, int64_t min_count, int32_t* dflt);
+
 /* ------------------------------------------------------------ (a)2 gradients */
 
 /* First/second derivatives per output (softmax reading R12, diagonal
@@ -153,9 +162,12 @@ gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* 
  * (§3.3; the paper's Alg. 2 body is missing.)
  * bins uint8 with ld = p->ld_bins and gbdtmo_bins_bytes() of storage; q from gbdtmo_grad;
  * hist / cnt: this level's buffers (gbdtmo_hist_bytes(level)); slot = node index within the
- * level (heap id - (2^level - 1)).  Slots not built are left untouched. */
+ * level (heap id - (2^level - 1)).  Slots not built are left untouched.
+ * dflt (may be NULL): per-feature default bins (gbdtmo_default_bins); rows in a feature's
+ * default bin are not accumulated and that bin's entries are left undefined until
+ * gbdtmo_find_split recovers them from the node totals. */
 gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
-                                const uint8_t* bins, const int32_t* q, void* state,
+                                const uint8_t* bins, const int32_t* dflt, const int32_t* q, void* state,
                                 int64_t* hist, int32_t* cnt);
 
 /* ------------------------------------- (a)4 subtraction + (a)5 split search */
@@ -171,9 +183,11 @@ gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t
  *     (0 if none): larger gain wins, ties -> smallest (f, b) (reading R16); the same key is
  *     max-reduced across GPUs.
  * nbins int32 [m] (local features); scales from gbdtmo_grad; keys uint64 [2^level] (out,
- * every slot written).  parent_hist / parent_cnt: level-1 buffers (ignored at level 0). */
+ * every slot written).  parent_hist / parent_cnt: level-1 buffers (ignored at level 0).
+ * dflt (may be NULL, must match gbdtmo_build_hist's): the default bin of every feature is
+ * recomputed as node total - sum of the other bins and written back to the node's histogram. */
 gbdtmo_status gbdtmo_find_split(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
-                                const int32_t* nbins, const float* scales, void* state,
+                                const int32_t* nbins, const int32_t* dflt, const float* scales, void* state,
                                 int64_t* hist, int32_t* cnt,
                                 const int64_t* parent_hist, const int32_t* parent_cnt,
                                 uint64_t* keys);
@@ -193,7 +207,7 @@ gbdtmo_status gbdtmo_find_split(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t
  * hist / cnt / parent_hist / parent_cnt as for gbdtmo_find_split (a derived winner's sums are
  * parent - sibling).  Every xchg word is written. */
 gbdtmo_status gbdtmo_split_record(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
-                                  const uint8_t* bins, const float* scales, void* state,
+                                  const uint8_t* bins, const int32_t* dflt, const float* scales, void* state,
                                   const int64_t* hist, const int32_t* cnt,
                                   const int64_t* parent_hist, const int32_t* parent_cnt,
                                   const uint64_t* keys, int64_t* xchg);

@@ -23,7 +23,7 @@ SYMBOLS = (
     "gbdtmo_launch_count", "gbdtmo_bins_bytes", "gbdtmo_bin_workspace_bytes", "gbdtmo_state_bytes",
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
-    "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export",
+    "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins",
 )
 
 
@@ -68,9 +68,10 @@ def lib():
             "gbdtmo_xchg_count": ([PP, C.POINTER(i64)], C.c_int),
             "gbdtmo_bin": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz], C.c_int),
             "gbdtmo_grad": ([P, PP, P, P, P, P, P], C.c_int),
-            "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P], C.c_int),
-            "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P], C.c_int),
-            "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
+            "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
             "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
@@ -164,17 +165,23 @@ class Context:
         self._check(lib().gbdtmo_grad(self._h, C.byref(p), _ptr(y), _ptr(pred), _ptr(q), _ptr(scales),
                                       _ptr(state)), "gbdtmo_grad")
 
-    def gbdtmo_build_hist(self, p, level, bins, q, state, hist, cnt):
-        self._check(lib().gbdtmo_build_hist(self._h, C.byref(p), level, _ptr(bins), _ptr(q), _ptr(state),
-                                            _ptr(hist), _ptr(cnt)), "gbdtmo_build_hist")
+    def gbdtmo_default_bins(self, bins, n, m, ld_bins, B, min_count, dflt):
+        self._check(lib().gbdtmo_default_bins(self._h, _ptr(bins), n, m, ld_bins, B, min_count, _ptr(dflt)),
+                    "gbdtmo_default_bins")
 
-    def gbdtmo_find_split(self, p, level, nbins, scales, state, hist, cnt, parent_hist, parent_cnt, keys):
-        self._check(lib().gbdtmo_find_split(self._h, C.byref(p), level, _ptr(nbins), _ptr(scales), _ptr(state),
-                                            _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
+    def gbdtmo_build_hist(self, p, level, bins, dflt, q, state, hist, cnt):
+        self._check(lib().gbdtmo_build_hist(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(q),
+                                            _ptr(state), _ptr(hist), _ptr(cnt)), "gbdtmo_build_hist")
+
+    def gbdtmo_find_split(self, p, level, nbins, dflt, scales, state, hist, cnt, parent_hist, parent_cnt, keys):
+        self._check(lib().gbdtmo_find_split(self._h, C.byref(p), level, _ptr(nbins), _ptr(dflt), _ptr(scales),
+                                            _ptr(state), _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
                                             _ptr(keys)), "gbdtmo_find_split")
 
-    def gbdtmo_split_record(self, p, level, bins, scales, state, hist, cnt, parent_hist, parent_cnt, keys, xchg):
-        self._check(lib().gbdtmo_split_record(self._h, C.byref(p), level, _ptr(bins), _ptr(scales), _ptr(state),
+    def gbdtmo_split_record(self, p, level, bins, dflt, scales, state, hist, cnt, parent_hist, parent_cnt, keys,
+                            xchg):
+        self._check(lib().gbdtmo_split_record(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(scales),
+                                              _ptr(state),
                                               _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
                                               _ptr(keys), _ptr(xchg)), "gbdtmo_split_record")
 

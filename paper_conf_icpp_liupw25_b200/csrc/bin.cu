@@ -212,6 +212,39 @@ __global__ void k_bin_apply(const float* __restrict__ X, int64_t n, int64_t ld_x
 
 inline int64_t sort_tiles(int64_t n) { return (n + kSortTile - 1) / kSortTile; }
 
+// dflt[f] = most frequent bin of feature f (ties: smallest).  One block per 8 features (one
+// aligned 8-byte load per row), per-feature shared counters.
+__global__ void __launch_bounds__(256) k_default_bins(const uint8_t* __restrict__ bins, int64_t n, int m, int64_t ld,
+                                                      int B, int64_t min_count, int32_t* __restrict__ dflt) {
+  __shared__ uint32_t c[8][256];
+  for (int i = threadIdx.x; i < 8 * 256; i += blockDim.x) (&c[0][0])[i] = 0;
+  __syncthreads();
+  const int f0 = blockIdx.x * 8;
+  for (int64_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const uint64_t w = *reinterpret_cast<const uint64_t*>(bins + i * ld + f0);
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      if (f0 + j < m) atomicAdd(&c[j][(w >> (8 * j)) & 0xFF], 1u);
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;   // warp j -> feature f0 + j
+  if (f0 + warp < m) {
+    uint32_t best = 0;
+    int bb = 0;
+    for (int b = lane; b < B; b += 32) {
+      const uint32_t v = c[warp][b];
+      if (v > best) { best = v; bb = b; }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const uint32_t ov = __shfl_xor_sync(0xffffffffu, best, o);
+      const int ob = __shfl_xor_sync(0xffffffffu, bb, o);
+      if (ov > best || (ov == best && ob < bb)) { best = ov; bb = ob; }
+    }
+    if (lane == 0) dflt[f0 + warp] = ((int64_t)best >= min_count) ? bb : -1;
+  }
+}
+
 }  // namespace gbdtmo
 
 using namespace gbdtmo;
@@ -257,5 +290,16 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
     GB_LAUNCH(k_bin_cuts, (unsigned)tc, 1024, 0, kin, n, B, cuts + (int64_t)c0 * (B - 1), nbins + c0);
     GB_LAUNCH(k_bin_apply, ctx->num_sms * 4, 256, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts, nbins, bins, ld_bins);
   }
+  return GBDTMO_OK;
+}
+
+extern "C" gbdtmo_status gbdtmo_default_bins(gbdtmo_ctx c, const uint8_t* bins, int64_t n, int32_t m, int64_t ld_bins,
+                                             int32_t B, int64_t min_count, int32_t* dflt) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  GB_CHECK_ARG(bins && dflt, "null pointer");
+  GB_CHECK_ARG(n >= 1 && m >= 1 && ld_bins >= m && ld_bins % 8 == 0 && B >= 2 && B <= 256, "bad shape");
+  GB_CHECK_ARG(((uintptr_t)bins & 7) == 0, "bins must be 8-byte aligned");
+  GB_LAUNCH(k_default_bins, (unsigned)((m + 7) / 8), 256, 0, bins, n, m, ld_bins, B, min_count, dflt);
   return GBDTMO_OK;
 }

@@ -71,9 +71,10 @@ __device__ __forceinline__ int byte_of_rt(const uint64_t (&sw)[SW], int j) {  //
 // shifts it, counts it (CNT) and parks the bins in the scratch; then the K groups of
 // 32/K rows are accumulated, lanes (row, channel) reading their bins back with one LDS and
 // their q value from a batch-wide prefetch.
-template <int K, int KF>
+template <int K, int KF, bool SKIP>
 __global__ void __launch_bounds__(kHistThreads, 1)
-k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ q,
+k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ dflt,
+            const int32_t* __restrict__ q,
             const int32_t* __restrict__ rows, int use_rows, State s,
             int64_t* __restrict__ hist, int32_t* __restrict__ cnt) {
   extern __shared__ __align__(16) uint32_t sm[];
@@ -110,6 +111,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int kk = min(KF, m - f0);
     const int c0 = ct * K;
     const bool do_cnt = (ct == 0);
+    int dfl[KF];                                   // default (skipped) bin per feature, -1: none
+#pragma unroll
+    for (int j = 0; j < KF; ++j) dfl[j] = (SKIP && j < kk) ? __ldg(&dflt[f0 + j]) : -1;
 
     const int words = limb_words + cnt_words;
     for (int i = threadIdx.x * 4; i < limb_words; i += blockDim.x * 4)
@@ -153,8 +157,10 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         shift_window<NW, SW>(w_cur, o, sw);
         if (do_cnt) {
 #pragma unroll
-          for (int j = 0; j < KF; ++j)
-            if (j < kk) red_shared_add(acnt + 4u * (j * B + byte_of<SW>(sw, j)), 1u);   // counts[j][b]: bank = b mod 32
+          for (int j = 0; j < KF; ++j) {
+            const uint32_t bin = byte_of<SW>(sw, j);
+            if (j < kk && (!SKIP || (int)bin != dfl[j])) red_shared_add(acnt + 4u * (j * B + bin), 1u);  // counts[j][b]
+          }
         }
       }
 #pragma unroll
@@ -183,14 +189,16 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #pragma unroll
               for (int j = 0; j < KF; ++j) {
                 const uint32_t bin = byte_of<SW>(bw, j);
-                red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-                red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+                if (!SKIP || (int)bin != dfl[j]) {
+                  red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+                  red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
+                }
               }
             } else {
 #pragma unroll
               for (int j = 0; j < KF; ++j) {
-                if (j < kk) {
-                  const uint32_t bin = byte_of<SW>(bw, j);
+                const uint32_t bin = byte_of<SW>(bw, j);
+                if (j < kk && (!SKIP || (int)bin != dfl[j])) {
                   red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
                   red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
                 }
@@ -253,33 +261,43 @@ __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __re
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += stride) cb[i] = 0;
 }
 
-template <int K, int KF>
-static gbdtmo_status launch_hist_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
-                                    const int32_t* q, const int32_t* rows, int use_rows, const State& s,
-                                    int64_t* hist, int32_t* cnt) {
+template <int K, int KF, bool SKIP>
+static gbdtmo_status launch_hist_kfs(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
+                                     const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows,
+                                     const State& s, int64_t* hist, int32_t* cnt) {
   static bool attr_done = false;
   if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_smem<K, KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin - 1024);
+    cudaFuncSetAttribute(k_hist_smem<K, KF, SKIP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         ctx->max_smem_optin - 1024);
     attr_done = true;
   }
-  GB_LAUNCH((k_hist_smem<K, KF>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+  GB_LAUNCH((k_hist_smem<K, KF, SKIP>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, dflt, q, rows, use_rows, s,
+            hist, cnt);
   return GBDTMO_OK;
+}
+
+template <int K, int KF>
+static gbdtmo_status launch_hist_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
+                                    const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows,
+                                    const State& s, int64_t* hist, int32_t* cnt) {
+  if (dflt) return launch_hist_kfs<K, KF, true>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  return launch_hist_kfs<K, KF, false>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
 }
 
 template <int K>
 static gbdtmo_status launch_hist(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
-                                 const int32_t* q, const int32_t* rows, int use_rows, const State& s,
+                                 const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows, const State& s,
                                  int64_t* hist, int32_t* cnt) {
   switch (hc.k) {
-    case 24: return launch_hist_kf<K, 24>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 16: return launch_hist_kf<K, 16>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 12: return launch_hist_kf<K, 12>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 8: return launch_hist_kf<K, 8>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 6: return launch_hist_kf<K, 6>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 4: return launch_hist_kf<K, 4>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 3: return launch_hist_kf<K, 3>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 2: return launch_hist_kf<K, 2>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    default: return launch_hist_kf<K, 1>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 24: return launch_hist_kf<K, 24>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 16: return launch_hist_kf<K, 16>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 12: return launch_hist_kf<K, 12>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 8: return launch_hist_kf<K, 8>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 6: return launch_hist_kf<K, 6>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 4: return launch_hist_kf<K, 4>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 3: return launch_hist_kf<K, 3>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 2: return launch_hist_kf<K, 2>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    default: return launch_hist_kf<K, 1>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
   }
 }
 
@@ -288,7 +306,7 @@ static gbdtmo_status launch_hist(Ctx* ctx, const gbdtmo_problem& p, const HistCf
 using namespace gbdtmo;
 
 extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
-                                           const uint8_t* bins, const int32_t* q, void* state,
+                                           const uint8_t* bins, const int32_t* dflt, const int32_t* q, void* state,
                                            int64_t* hist, int32_t* cnt) {
   Ctx* ctx = (Ctx*)c;
   if (!ctx) return GBDTMO_EINVAL;
@@ -306,8 +324,8 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
   const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
   const int use_rows = level > 0;
   switch (hc.K) {
-    case 4: return launch_hist<4>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    case 8: return launch_hist<8>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
-    default: return launch_hist<16>(ctx, *p, hc, bins, q, rows, use_rows, s, hist, cnt);
+    case 4: return launch_hist<4>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 8: return launch_hist<8>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    default: return launch_hist<16>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
   }
 }

@@ -29,8 +29,8 @@ __device__ __forceinline__ long long warp_excl(long long x, long long* total) {
   return v - x;
 }
 
-// 8 consecutive int64 bins [8 lane, 8 lane + 8) of one channel row (bins contiguous), for a
-// derived node parent - sibling (written back when `store`); inclusive in-lane prefix on return.
+// 8 consecutive int64 bins [8 lane, 8 lane + 8) of one channel row (raw values; for a derived
+// node parent - sibling, written back when `store`).
 __device__ __forceinline__ void load_row8(long long (&v)[kFsBins], const int64_t* cur, const int64_t* par,
                                           const int64_t* sib, bool derive, bool store, int B) {
   const int lane = threadIdx.x & 31;
@@ -63,18 +63,44 @@ __device__ __forceinline__ void load_row8(long long (&v)[kFsBins], const int64_t
       v[i] = x;
     }
   }
+}
+
+// Inclusive prefix over bins of one row held 8 bins per lane.  The default bin `db` (sparsity-
+// aware skip; -1: none) is not trusted: its value is recovered as node total - sum of the other
+// bins, written back through `wb` when non-null.  Returns the node total.
+__device__ __forceinline__ long long row_prefix(long long (&v)[kFsBins], int db, long long node_total,
+                                                int64_t* wb, long long* delta_out = nullptr) {
+  const int lane = threadIdx.x & 31;
+  const int b0 = lane * kFsBins;
+  const bool mine = db >= b0 && db < b0 + kFsBins;
+#pragma unroll
+  for (int i = 0; i < kFsBins; ++i) if (mine && db == b0 + i) v[i] = 0;
 #pragma unroll
   for (int i = 1; i < kFsBins; ++i) v[i] += v[i - 1];
+  long long others;
+  const long long ex = warp_excl(v[kFsBins - 1], &others);
+  if (db < 0) {
+#pragma unroll
+    for (int i = 0; i < kFsBins; ++i) v[i] += ex;
+    return others;
+  }
+  const long long delta = node_total - others;
+#pragma unroll
+  for (int i = 0; i < kFsBins; ++i) v[i] += ex + ((b0 + i >= db) ? delta : 0);
+  if (mine && wb) wb[db] = delta;
+  if (delta_out) *delta_out = delta;
+  return node_total;
 }
 
 // One warp per (node, feature); lane l owns bins [8l, 8l + 8).  Per channel the warp reads the
 // contiguous row of B int64 bins (channel-major histogram: coalesced 16-byte loads), prefix-sums
-// it (in-lane + warp scan), and accumulates per bin: MSE sum_k G_L^2 and sum_k G_R^2 (H = 2 C is
-// shared by all outputs: two divisions per bin), softmax the Eq. (3) terms.
+// it (in-lane + warp scan; the feature's default bin recovered from the exact node totals), and
+// accumulates per bin: MSE sum_k G_L^2 and sum_k G_R^2 (H = 2 C is shared by all outputs: two
+// divisions per bin), softmax the Eq. (3) terms.
 template <bool SOFTMAX>
 __global__ void __launch_bounds__(kFsWarps * 32)
-k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
-             State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt,
+k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const int32_t* __restrict__ dflt,
+             const float* __restrict__ scales, State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt,
              const int64_t* __restrict__ phist, const int32_t* __restrict__ pcnt,
              uint64_t* __restrict__ keys, int write_derived) {
   const int slot = blockIdx.y;
@@ -82,19 +108,23 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   if (s.node_state[h] != GBDTMO_NODE_ACTIVE) return;
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const bool store = derive && write_derived;
+  const bool own = !derive || store;                  // this node's histogram may be written
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int f = blockIdx.x * kFsWarps + warp;
   const int sib = slot ^ 1, par = slot >> 1;
   const double lam = p.lambda;
+  const int64_t* S = s.node_sum + h * (V + 1);         // exact node totals (channels, count)
   __shared__ unsigned long long wbest[kFsWarps];
   uint64_t best = 0;
   if (f < m) {
+    const int db = dflt ? dflt[f] : -1;
+    const int b0 = lane * kFsBins;
     // counts
     long long cl[kFsBins];
+    long long ctot;
     {
       const int64_t oc = ((int64_t)slot * m + f) * B, os = ((int64_t)sib * m + f) * B, op = ((int64_t)par * m + f) * B;
-      const int b0 = lane * kFsBins;
 #pragma unroll
       for (int i = 0; i < kFsBins; ++i) {
         const int b = b0 + i;
@@ -105,71 +135,65 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
         }
         cl[i] = x;
       }
+      long long dc = 0;
+      ctot = row_prefix(cl, db, S[V], nullptr, &dc);
+      if (own && db >= b0 && db < b0 + kFsBins) cnt[oc + db] = (int32_t)dc;   // recovered default-bin count
+    }
+    // ---- channels
+    const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
+                  rowp = ((int64_t)par * m + f) * V * B;
+    double accL[kFsBins], accR[kFsBins];
 #pragma unroll
-      for (int i = 1; i < kFsBins; ++i) cl[i] += cl[i - 1];
-      long long ctot;
-      const long long ex = warp_excl(cl[kFsBins - 1], &ctot);
+    for (int i = 0; i < kFsBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
+    double P = 0.0;
+    for (int k = 0; k < d; ++k) {
+      long long gv[kFsBins];
+      int64_t* rg = hist + rowc + (int64_t)k * B;
+      load_row8(gv, rg, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B, derive, store, B);
+      const long long G = row_prefix(gv, db, S[k], own ? rg : nullptr);
+      const double sg = (double)scales[k];
+      if (!SOFTMAX) {
 #pragma unroll
-      for (int i = 0; i < kFsBins; ++i) cl[i] += ex;
-      cl[0] = cl[0];  // (keeps the array in registers)
-      // ---- channels
-      const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
-                    rowp = ((int64_t)par * m + f) * V * B;
-      double accL[kFsBins], accR[kFsBins];
-#pragma unroll
-      for (int i = 0; i < kFsBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
-      double P = 0.0;
-      for (int k = 0; k < d; ++k) {
-        long long gv[kFsBins];
-        load_row8(gv, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
-                  derive, store, B);
-        long long G;
-        const long long gex = warp_excl(gv[kFsBins - 1], &G);
-        const double sg = (double)scales[k];
-        if (!SOFTMAX) {
-#pragma unroll
-          for (int i = 0; i < kFsBins; ++i) {
-            const double GL = (double)(gv[i] + gex) * sg, GR = (double)(G - gv[i] - gex) * sg;
-            accL[i] = fma(GL, GL, accL[i]);
-            accR[i] = fma(GR, GR, accR[i]);
-          }
-          const double Gd = (double)G * sg;
-          P = fma(Gd, Gd, P);
-        } else {
-          long long hv[kFsBins];
-          load_row8(hv, hist + rowc + (int64_t)(d + k) * B, phist + rowp + (int64_t)(d + k) * B,
-                    hist + rows_ + (int64_t)(d + k) * B, derive, store, B);
-          long long H;
-          const long long hex = warp_excl(hv[kFsBins - 1], &H);
-          const double sh = (double)scales[d + k];
-#pragma unroll
-          for (int i = 0; i < kFsBins; ++i) {
-            const double GL = (double)(gv[i] + gex) * sg, GR = (double)(G - gv[i] - gex) * sg;
-            const double HL = (double)(hv[i] + hex) * sh, HR = (double)(H - hv[i] - hex) * sh;
-            accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
-          }
-          const double Gd = (double)G * sg, Hd = (double)H * sh;
-          P += Gd * Gd / (Hd + lam);
+        for (int i = 0; i < kFsBins; ++i) {
+          const double GL = (double)gv[i] * sg, GR = (double)(G - gv[i]) * sg;
+          accL[i] = fma(GL, GL, accL[i]);
+          accR[i] = fma(GR, GR, accR[i]);
         }
-      }
-      // ---- gains and the lane's best candidate
-      const int nb = nbins[f];
-      const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
+        const double Gd = (double)G * sg;
+        P = fma(Gd, Gd, P);
+      } else {
+        long long hv[kFsBins];
+        int64_t* rh = hist + rowc + (int64_t)(d + k) * B;
+        load_row8(hv, rh, phist + rowp + (int64_t)(d + k) * B, hist + rows_ + (int64_t)(d + k) * B, derive, store, B);
+        const long long H = row_prefix(hv, db, S[d + k], own ? rh : nullptr);
+        const double sh = (double)scales[d + k];
 #pragma unroll
-      for (int i = 0; i < kFsBins; ++i) {
-        const int b = b0 + i;
-        const long long c = cl[i];
-        if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
-          double gain;
-          if (!SOFTMAX)
-            gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
-                          P / (2.0 * (double)ctot + lam));
-          else
-            gain = 0.5 * (accL[i] - P);
-          if (gain > p.gamma) {
-            const uint64_t key = pack_key(gain, fb0 + b);
-            best = key > best ? key : best;
-          }
+        for (int i = 0; i < kFsBins; ++i) {
+          const double GL = (double)gv[i] * sg, GR = (double)(G - gv[i]) * sg;
+          const double HL = (double)hv[i] * sh, HR = (double)(H - hv[i]) * sh;
+          accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+        }
+        const double Gd = (double)G * sg, Hd = (double)H * sh;
+        P += Gd * Gd / (Hd + lam);
+      }
+    }
+    // ---- gains and the lane's best candidate
+    const int nb = nbins[f];
+    const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
+#pragma unroll
+    for (int i = 0; i < kFsBins; ++i) {
+      const int b = b0 + i;
+      const long long c = cl[i];
+      if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
+        double gain;
+        if (!SOFTMAX)
+          gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
+                        P / (2.0 * (double)ctot + lam));
+        else
+          gain = 0.5 * (accL[i] - P);
+        if (gain > p.gamma) {
+          const uint64_t key = pack_key(gain, fb0 + b);
+          best = key > best ? key : best;
         }
       }
     }
@@ -204,7 +228,8 @@ __device__ __forceinline__ bool decode_local(const gbdtmo_problem& p, uint64_t k
 }
 
 // One block per slot: left sums at the winning (feature, bin) if the feature is local.
-__global__ void k_split_record(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ hist,
+__global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __restrict__ dflt, State s,
+                               const int64_t* __restrict__ hist,
                                const int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
                                const int32_t* __restrict__ pcnt, const uint64_t* __restrict__ keys,
                                const float* __restrict__ scales, int64_t* __restrict__ xchg) {
@@ -223,19 +248,28 @@ __global__ void k_split_record(gbdtmo_problem p, int level, State s, const int64
   const int sib = slot ^ 1, par = slot >> 1;
   const int64_t rc = ((int64_t)slot * m + fl) * B, rs = ((int64_t)sib * m + fl) * B, rp = ((int64_t)par * m + fl) * B;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  for (int c = warp; c < V; c += nw) {          // hist is [slot][f][c][b]: a warp sums bins <= b of channel c
-    long long acc = 0;
-    for (int bb = lane; bb <= b; bb += 32)
-      acc += derive ? (phist[(rp * V) + (int64_t)c * B + bb] - hist[(rs * V) + (int64_t)c * B + bb])
-                    : hist[(rc * V) + (int64_t)c * B + bb];
+  const int db = dflt ? dflt[fl] : -1;            // default bin: recovered from the node totals
+  const int64_t* S = s.node_sum + h * (V + 1);
+  for (int c = warp; c <= V; c += nw) {           // c == V: the counts
+    long long le = 0, all = 0;
+    for (int bb = lane; bb < B; bb += 32) {
+      if (bb == db) continue;
+      long long x;
+      if (c < V) x = derive ? (phist[(rp * V) + (int64_t)c * B + bb] - hist[(rs * V) + (int64_t)c * B + bb])
+                            : hist[(rc * V) + (int64_t)c * B + bb];
+      else x = derive ? (long long)(pcnt[rp + bb] - cnt[rs + bb]) : (long long)cnt[rc + bb];
+      all += x;
+      if (bb <= b) le += x;
+    }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (lane == 0) rec[c] = acc;
+    for (int o = 16; o > 0; o >>= 1) {
+      le += __shfl_xor_sync(0xffffffffu, le, o);
+      all += __shfl_xor_sync(0xffffffffu, all, o);
+    }
+    if (db >= 0 && db <= b) le += S[c] - all;      // (S[V] = the node's row count)
+    if (lane == 0) rec[c] = le;
   }
   if (threadIdx.x == 0) {
-    long long cl = 0;
-    for (int bb = 0; bb <= b; ++bb) cl += derive ? (pcnt[rp + bb] - cnt[rs + bb]) : cnt[rc + bb];
-    rec[V] = cl;
     rec[V + 1] = fg + 1;
     rec[V + 2] = b;
   }
@@ -244,7 +278,6 @@ __global__ void k_split_record(gbdtmo_problem p, int level, State s, const int64
     // exact Eq. (3) at the winner from the exact sums (informational: the tree record's gain)
     const int d = p.d;
     const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
-    const int64_t* S = s.node_sum + h * (V + 1);
     const long long ctot = S[V], cl = rec[V];
     double g = 0.0;
     for (int k = 0; k < d; ++k) {
@@ -300,7 +333,7 @@ __global__ void k_bitmap(gbdtmo_problem p, int level, const uint8_t* __restrict_
 using namespace gbdtmo;
 
 extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
-                                           const int32_t* nbins, const float* scales, void* state,
+                                           const int32_t* nbins, const int32_t* dflt, const float* scales, void* state,
                                            int64_t* hist, int32_t* cnt, const int64_t* parent_hist,
                                            const int32_t* parent_cnt, uint64_t* keys) {
   Ctx* ctx = (Ctx*)c;
@@ -315,13 +348,13 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
   dim3 grid((p->m + kFsWarps - 1) / kFsWarps, (unsigned)LN);
   auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_find_split<true> : k_find_split<false>;
-  GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt,
+  GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, dflt, scales, s, hist, cnt,
             level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
   return GBDTMO_OK;
 }
 
 extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
-                                             const uint8_t* bins, const float* scales, void* state,
+                                             const uint8_t* bins, const int32_t* dflt, const float* scales, void* state,
                                              const int64_t* hist, const int32_t* cnt,
                                              const int64_t* parent_hist, const int32_t* parent_cnt,
                                              const uint64_t* keys, int64_t* xchg) {
@@ -334,7 +367,7 @@ extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem*
   GB_CHECK_ARG(level == 0 || (parent_hist && parent_cnt), "parent histogram required for level > 0");
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
-  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, s, hist, cnt, level > 0 ? parent_hist : hist,
+  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, s, hist, cnt, level > 0 ? parent_hist : hist,
             level > 0 ? parent_cnt : cnt, keys, scales, xchg);
   // zero the record words of the unused slots of this buffer (levels < D-1) so SUM-merging is clean
   const int64_t used = LN * rec_words(*p), cap = bitmap_offset(*p);

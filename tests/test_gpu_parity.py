@@ -126,7 +126,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
     rows = node_rows(bins, ref["state"][0], ref["feat"][0], ref["bin"][0], w.n)
     g, h = orc.grad(w.loss, Y.astype(np.float64), np.zeros(Y.shape))
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1))
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1), sparse_default=True)
     ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
     ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
     sc = None
@@ -165,15 +165,17 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------- whole trees
 
-@pytest.mark.parametrize("case", ["C1", "C2s", "C3s", "C4s", "C5s"])
-def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case):
+@pytest.mark.parametrize("case,sparse", [("C1", False), ("C2s", False), ("C2s", True), ("C3s", False),
+                                         ("C4s", False), ("C5s", False)])
+def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse):
     w = CASES[case]
     X, Y = _inputs(w)
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
     ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
                     lr=w.lr, min_node=w.min_node)
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w))
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse)
+    assert (b.dflt is not None) == (sparse and w.index == 2)     # only the MNIST-shaped data has dominant bins
     b.fit()
     torch.cuda.synchronize()
     for t in range(w.T):
@@ -239,15 +241,15 @@ def test_two_shards_equal_one(orc, pkg, ctx):
             for s in shards:
                 ph = s.hist[par] if lvl else None
                 pc = s.cnt[par] if lvl else None
-                ctx.gbdtmo_build_hist(s.p, lvl, s.ds.bins, s.q, s.state, s.hist[cur], s.cnt[cur])
-                ctx.gbdtmo_find_split(s.p, lvl, s.ds.nbins, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
+                ctx.gbdtmo_build_hist(s.p, lvl, s.ds.bins, s.dflt, s.q, s.state, s.hist[cur], s.cnt[cur])
+                ctx.gbdtmo_find_split(s.p, lvl, s.ds.nbins, s.dflt, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
                                       s.keys)
             kmax = torch.maximum(shards[0].keys, shards[1].keys)
             for s in shards:
                 s.keys.copy_(kmax)
                 ph = s.hist[par] if lvl else None
                 pc = s.cnt[par] if lvl else None
-                ctx.gbdtmo_split_record(s.p, lvl, s.ds.bins, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
+                ctx.gbdtmo_split_record(s.p, lvl, s.ds.bins, s.dflt, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
                                         s.keys, s.xchg)
             xs = shards[0].xchg + shards[1].xchg
             for s in shards:

@@ -240,10 +240,23 @@ gbdtmo_status gbdtmo_update_pred(gbdtmo_ctx ctx, const gbdtmo_problem* p, const 
 
 /* Copy of the tree record (heap-indexed, 2^(D+1)-1 entries each) out of `state`:
  * node_state (GBDTMO_NODE_*), feature (global id, -1 if none), bin, gain (fp64),
- * n_rows, n_left.  Any output pointer may be NULL. */
+ * n_rows, n_left, and threshold = cuts[f][bin] (float32, x < threshold goes left, reading R15)
+ * for split features held by this process (0 elsewhere: a SUM across processes merges them).
+ * cuts: gbdtmo_bin's [m][B-1] of the local features (may be NULL when threshold is NULL).
+ * Any output pointer may be NULL. */
 gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx ctx, const gbdtmo_problem* p, const void* state,
                                  int32_t* node_state, int32_t* feature, int32_t* bin, double* gain,
-                                 int64_t* n_rows, int64_t* n_left);
+                                 int64_t* n_rows, int64_t* n_left, const float* cuts, float* threshold);
+
+/* Inference for unseen instances (instance-level parallelism):
+ * for every row i and tree t = 0..T-1 in order, walk from the root: at a SPLIT node go left iff
+ * X[i][feature] < threshold, at a LEAF add its value:  pred[i][k] += leaf[t][h][k].
+ * X float32 row-major [n][ld_x] over ALL (global) features; node_state / feature int32 [T][NH],
+ * threshold float32 [T][NH], leaf float64 [T][NH][d] as exported per tree (NH = 2^(D+1)-1);
+ * pred float64 [n][d] in/out (start from zeros for a fresh prediction). */
+gbdtmo_status gbdtmo_predict(gbdtmo_ctx ctx, const float* X, int64_t n, int64_t ld_x, int32_t T, int32_t D,
+                             int32_t d, const int32_t* node_state, const int32_t* feature,
+                             const float* threshold, const double* leaf, double* pred);
 
 /* Copy of the row bookkeeping out of `state` (tests, debugging): the row-index list as seen by
  * `level` (level = D: after the last partition), int32 [n]; the heap node of every instance,

@@ -23,7 +23,7 @@ SYMBOLS = (
     "gbdtmo_launch_count", "gbdtmo_bins_bytes", "gbdtmo_bin_workspace_bytes", "gbdtmo_state_bytes",
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
-    "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins",
+    "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
 )
 
 
@@ -75,7 +75,8 @@ def lib():
             "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
             "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
-            "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_predict": ([P, P, i64, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
             "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
         }
         for name, (args, res) in sig.items():
@@ -198,10 +199,14 @@ class Context:
                     "gbdtmo_update_pred")
 
     def gbdtmo_tree_export(self, p, state, node_state=None, feature=None, bin=None, gain=None, n_rows=None,
-                           n_left=None):
+                           n_left=None, cuts=None, threshold=None):
         self._check(lib().gbdtmo_tree_export(self._h, C.byref(p), _ptr(state), _ptr(node_state), _ptr(feature),
-                                             _ptr(bin), _ptr(gain), _ptr(n_rows), _ptr(n_left)),
-                    "gbdtmo_tree_export")
+                                             _ptr(bin), _ptr(gain), _ptr(n_rows), _ptr(n_left), _ptr(cuts),
+                                             _ptr(threshold)), "gbdtmo_tree_export")
+
+    def gbdtmo_predict(self, X, n, ld_x, T, D, d, node_state, feature, threshold, leaf, pred):
+        self._check(lib().gbdtmo_predict(self._h, _ptr(X), n, ld_x, T, D, d, _ptr(node_state), _ptr(feature),
+                                         _ptr(threshold), _ptr(leaf), _ptr(pred)), "gbdtmo_predict")
 
     def gbdtmo_rows_export(self, p, state, level, rows=None, node_of_row=None, node_begin=None, node_end=None):
         self._check(lib().gbdtmo_rows_export(self._h, C.byref(p), _ptr(state), level, _ptr(rows), _ptr(node_of_row),

@@ -166,9 +166,12 @@ class Booster:
                    bin=torch.empty(NH, dtype=torch.int32, device=dev),
                    gain=torch.empty(NH, dtype=torch.float64, device=dev),
                    n_rows=torch.empty(NH, dtype=torch.int64, device=dev),
-                   n_left=torch.empty(NH, dtype=torch.int64, device=dev))
+                   n_left=torch.empty(NH, dtype=torch.int64, device=dev),
+                   threshold=torch.empty(NH, dtype=torch.float32, device=dev))
         self.ctx.gbdtmo_tree_export(self.p, self.state, rec["node_state"], rec["feature"], rec["bin"], rec["gain"],
-                                    rec["n_rows"], rec["n_left"])
+                                    rec["n_rows"], rec["n_left"], self.ds.cuts, rec["threshold"])
+        if self.group is not None:   # thresholds live with the feature's owner: SUM merges them
+            parallel.exchange_records(rec["threshold"], self.group)
         rec["leaf"] = self.leaf.clone()
         return rec
 
@@ -213,3 +216,22 @@ def train(X, Y, params: Params, device: str = "cuda:0", ctx: Optional[Context] =
     b = Booster(ctx, ds, Yd, params, group=group)
     b.fit()
     return b
+
+
+def predict(ctx: Context, trees, X: torch.Tensor, D: int, d: int, pred: Optional[torch.Tensor] = None):
+    """gbdtmo_predict: sum of the trees' leaf values for unseen rows X (device float32 [n][m_global]).
+    `trees` is a list of exported tree records (Booster.trees)."""
+    assert X.is_cuda and X.dtype == torch.float32 and X.stride(1) == 1
+    n = X.shape[0]
+    T = len(trees)
+    dev = X.device
+    pred = pred if pred is not None else torch.zeros((n, d), dtype=torch.float64, device=dev)
+    if T == 0:
+        return pred
+    st = torch.stack([t["node_state"] for t in trees]).contiguous()
+    ft = torch.stack([t["feature"] for t in trees]).contiguous()
+    th = torch.stack([t["threshold"] for t in trees]).contiguous()
+    lf = torch.stack([t["leaf"] for t in trees]).contiguous()
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
+    ctx.gbdtmo_predict(X, n, X.stride(0), T, D, d, st, ft, th, lf, pred)
+    return pred

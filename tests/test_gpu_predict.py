@@ -1,0 +1,61 @@
+"""Inference for unseen rows through gbdtmo_predict."""
+import numpy as np
+import pytest
+import torch
+
+from gen import gen
+
+pytestmark = pytest.mark.gpu
+
+
+def _host_predict(X, cuts, trees, D, d):
+    """Reference walk (test harness): x < cuts[f][b] goes left (reading R15)."""
+    n = X.shape[0]
+    NH = (1 << (D + 1)) - 1
+    out = np.zeros((n, d))
+    for t in range(trees["state"].shape[0]):
+        st, ft, bt, lv = trees["state"][t], trees["feat"][t], trees["bin"][t], trees["leaf"][t]
+        h = np.zeros(n, np.int64)
+        for _ in range(D + 1):
+            s = st[h] == 1
+            if not s.any():
+                break
+            f, b = ft[h[s]], bt[h[s]]
+            go_left = X[np.nonzero(s)[0], f] < cuts[f, b]
+            h[s] = np.where(go_left, 2 * h[s] + 1, 2 * h[s] + 2)
+        assert np.all(st[h] == 2)
+        out += lv[h]
+        assert h.max() < NH
+    return out
+
+
+@pytest.mark.parametrize("case", ["C1", "C3s", "C2s"])
+def test_predict_train_rows_equals_training_prediction_and_oracle_on_unseen(orc, case):
+    import paper_conf_icpp_liupw25_b200 as pkg
+    w = {"C1": gen.WORKLOADS["C1"], "C3s": gen.WORKLOADS["C3"].scaled(n=50_000, m=20, T=3, D=6),
+         "C2s": gen.WORKLOADS["C2"].scaled(n=20_000, m=64, T=3, D=5)}[case]
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    ctx = pkg.Context(0)
+    P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P)
+    b.fit()
+    # training rows: the instance-parallel walk reproduces the incremental training prediction exactly
+    pt = pkg.predict(ctx, b.trees, torch.from_numpy(X).cuda(), w.D, w.d)
+    torch.cuda.synchronize()
+    assert torch.equal(pt, b.pred)
+    # unseen rows (next row range of the same generator) vs the oracle's trees walked on the host
+    Xu = gen.features_host(w, r0=w.n, nr=7_000)
+    pu = pkg.predict(ctx, b.trees, torch.from_numpy(Xu).cuda(), w.D, w.d).cpu().numpy()
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    hu = _host_predict(Xu, cuts, dict(state=ref["state"], feat=ref["feat"], bin=ref["bin"], leaf=ref["leaf"]),
+                       w.D, w.d)
+    assert np.max(np.abs(pu - hu)) <= 1e-4
+    # and the exported thresholds are the oracle's cut values
+    for t in range(w.T):
+        st = b.trees[t]["node_state"].cpu().numpy()
+        thr = b.trees[t]["threshold"].cpu().numpy()
+        sp = st == 1
+        np.testing.assert_array_equal(thr[sp], cuts[ref["feat"][t][sp], ref["bin"][t][sp]])

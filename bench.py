@@ -148,7 +148,7 @@ def cpu_oracle_sample(w, feats=128, trees=1):
     cols = np.linspace(0, w.m - 1, feats).astype(np.int64)
     X = np.empty((w.n, feats), np.float32)
     for j, c in enumerate(cols):
-        X[:, j] = gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, int(c), 1, w.m)[:, 0]
+        X[:, j] = gen.features_host(w, 0, w.n, int(c), 1)[:, 0]
     Y = host_targets(w).astype(np.float64)
     cuts, nbins, bins = oracle.bin_matrix(X, w.B)
     del X
@@ -175,7 +175,7 @@ def main():
     a = parse()
     rank, world, local = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1), _env_int("LOCAL_RANK", 0)
     from gen import gen
-    w = gen.WORKLOADS[a.workload]
+    w = gen.sweep(int(a.workload[1:])) if a.workload.startswith("S") else gen.WORKLOADS[a.workload]
 
     if a.impl == "reference":
         if rank != 0:
@@ -220,9 +220,12 @@ def main():
     t_setup = time.perf_counter()
     Yh = host_targets(w)
     Y = torch.from_numpy(Yh).to(dev)
-    X = torch.empty((w.n, m_loc), dtype=torch.float32, device=dev)
-    gen.matrix_cuda(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, X.data_ptr(), m_loc,
-                    torch.cuda.current_stream().cuda_stream)
+    if w.classes_sweep:                 # features depend on the labels: generated on the host
+        X = torch.from_numpy(gen.features_host(w, 0, w.n, f0, m_loc)).to(dev)
+    else:
+        X = torch.empty((w.n, m_loc), dtype=torch.float32, device=dev)
+        gen.matrix_cuda(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, X.data_ptr(), m_loc,
+                        torch.cuda.current_stream().cuda_stream)
     torch.cuda.synchronize()
     tb0 = torch.cuda.Event(enable_timing=True); tb1 = torch.cuda.Event(enable_timing=True)
     tb0.record()
@@ -357,7 +360,8 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1):
     from gen import gen
     m_loc = f1 - f0
     Xh = torch.empty((w.n, m_loc), dtype=torch.float32, pin_memory=True)
-    gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, out=Xh.numpy())
+    Xh.numpy()[:] = gen.features_host(w, 0, w.n, f0, m_loc) if w.classes_sweep else \
+        gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, out=Xh.numpy())
     Yh = torch.from_numpy(host_targets(w)).pin_memory()
     ctx = pkg.Context(local)
     params = pkg.Params(loss=w.loss, T=a.steps, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,

@@ -110,6 +110,7 @@ class Workload:
     gamma: float = 0.0
     lr: float = 1.0
     min_node: int = 20
+    classes_sweep: bool = False      # NEXT-2 (Fig. 6b): sklearn-style multi-class, features depend on labels
 
     @property
     def seed(self):
@@ -128,6 +129,20 @@ WORKLOADS = {
 }
 
 
+def sweep(d: int, n: int = 100_000, m: int = 100, T: int = 100, D: int = 6) -> Workload:
+    """NEXT-2 class-count sweep (Fig. 6b: 100 trees of depth 6 on scikit-learn-style
+    multi-class data, 5..500 classes; DESIGN.md Inputs: n = 100k, m = 100, 20 informative features)."""
+    return Workload(f"S{d}-class-sweep", 100 + d, n, m, d, 256, D, T, LOSS_SOFTMAX, KIND_NORMAL, classes_sweep=True)
+
+
+def _sweep_labels(w: Workload, r0: int, nr: int):
+    return (np.floor(uniform_host(w.seed, STREAM_LABEL, r0, nr) * w.d)).astype(np.int64)
+
+
+def _sweep_centroids(w: Workload):
+    return 1.5 * normal_host(w.seed, STREAM_W, (w.d, 20))
+
+
 def informative_columns(w: Workload):
     """Columns the targets depend on (DESIGN.md Inputs)."""
     if w.index == 5:
@@ -140,7 +155,14 @@ def informative_columns(w: Workload):
 def features_host(w: Workload, r0=0, nr=None, c0=0, nc=None):
     nr = w.n - r0 if nr is None else nr
     nc = w.m - c0 if nc is None else nc
-    return matrix_host(w.seed, STREAM_X, w.x_kind, r0, nr, c0, nc, w.m)
+    X = matrix_host(w.seed, STREAM_X, w.x_kind, r0, nr, c0, nc, w.m)
+    if w.classes_sweep:            # class centroid shift on the 20 informative columns
+        lab = _sweep_labels(w, r0, nr)
+        cen = _sweep_centroids(w)
+        lo, hi = max(c0, 0), min(c0 + nc, 20)
+        if lo < hi:
+            X[:, lo - c0:hi - c0] += cen[lab][:, lo:hi].astype(np.float32)
+    return X
 
 
 def _columns_host(w: Workload, cols):
@@ -153,6 +175,10 @@ def _columns_host(w: Workload, cols):
 def targets_host(w: Workload, X=None):
     """Targets y [n][d] float32 (fp64-computed, rounded as stated in DESIGN.md Inputs)."""
     n, d = w.n, w.d
+    if w.classes_sweep:
+        y = np.zeros((n, d), np.float32)
+        y[np.arange(n), _sweep_labels(w, 0, n)] = 1.0
+        return y
     if w.index == 2:   # MNIST-shaped: label = argmax(X V / 255 + Gumbel); one-hot
         Xf = X if X is not None else features_host(w)
         V = normal_host(w.seed, STREAM_W, (w.m, d))

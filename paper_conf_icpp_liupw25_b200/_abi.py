@@ -11,7 +11,8 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgbdtmo.so")
+# GBDTMO_LIB overrides the library path (A/B builds of the same sources; see tools/ab_build.sh)
+LIB_PATH = os.environ.get("GBDTMO_LIB") or os.path.join(_HERE, "libgbdtmo.so")
 
 OK, EINVAL, ECUDA, ENOMEM, EUNSUPPORTED = 0, 1, 2, 3, 5
 LOSS_MSE, LOSS_SOFTMAX = 0, 1

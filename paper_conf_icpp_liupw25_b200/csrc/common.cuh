@@ -46,7 +46,10 @@ constexpr int kQShift = 30;            // q = rint(g * 2^30 / P), |q| <= 2^30
 constexpr int kChunkMax = 65536;       // rows per histogram work item: lo-limb sums < 2^32
 constexpr int kChunkMin = 512;
 constexpr int kPartTile = 2048;        // positions per partition block
-constexpr int kHistThreads = 1024;     // histogram CTA (1 CTA / SM, ~200 KB smem)
+#ifndef GBDTMO_HIST_THREADS
+#define GBDTMO_HIST_THREADS 1024
+#endif
+constexpr int kHistThreads = GBDTMO_HIST_THREADS;   // histogram CTA (1 CTA / SM, ~200 KB smem)
 constexpr int kHistSmemBudget = 218 * 1024;   // limbs + counts + per-warp row scratch
 constexpr int kHistWarps = kHistThreads / 32;
 constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte bin window)

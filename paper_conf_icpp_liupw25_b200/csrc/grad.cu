@@ -76,64 +76,55 @@ __global__ void k_mse_quantize(gbdtmo_problem p, const float* __restrict__ y, co
 }
 
 // Softmax (fp64): one warp per row; p = softmax(yhat) (max-subtracted), g = p - y, h = p (1 - p);
-// q_g = rint(g 2^30) (P = 1), q_h = rint(h 2^32) (P = 1/4).  d <= 256.
+// q_g = rint(g 2^30) (P = 1), q_h = rint(h 2^32) (P = 1/4).  Any d (lanes stride the outputs;
+// exp is recomputed instead of held in registers).
 __global__ void k_softmax_quantize(gbdtmo_problem p, const float* __restrict__ y, const double* __restrict__ pred,
                                    int32_t* __restrict__ q, float* __restrict__ scales, State s) {
-  constexpr int J = 8;  // channels per lane: d <= 32 * J
   const int d = p.d, V = 2 * d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  long long accg[J], acch[J];
-#pragma unroll
-  for (int j = 0; j < J; ++j) { accg[j] = 0; acch[j] = 0; }
   for (int64_t i = blockIdx.x * (int64_t)nw + warp; i < p.n; i += (int64_t)gridDim.x * nw) {
-    double z[J];
+    const double* pr = pred + i * d;
     double mx = -INFINITY;
-#pragma unroll
-    for (int j = 0; j < J; ++j) {
-      const int c = lane + 32 * j;
-      z[j] = c < d ? pred[i * d + c] : -INFINITY;
-      mx = fmax(mx, z[j]);
-    }
+    for (int c = lane; c < d; c += 32) mx = fmax(mx, pr[c]);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
     double sum = 0.0;
-#pragma unroll
-    for (int j = 0; j < J; ++j) {
-      const int c = lane + 32 * j;
-      z[j] = c < d ? exp(z[j] - mx) : 0.0;
-      sum += z[j];
-    }
+    for (int c = lane; c < d; c += 32) sum += exp(pr[c] - mx);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
-#pragma unroll
-    for (int j = 0; j < J; ++j) {
-      const int c = lane + 32 * j;
-      if (c < d) {
-        const double pr = z[j] / sum;
-        const double g = pr - (double)y[i * d + c];
-        const double h = pr * (1.0 - pr);
-        const int qg = __double2int_rn(ldexp(g, kQShift));
-        const int qh = __double2int_rn(ldexp(h, kQShift + 2));
-        q[i * V + c] = qg;
-        q[i * V + d + c] = qh;
-        accg[j] += qg;
-        acch[j] += qh;
-      }
-    }
-  }
-#pragma unroll
-  for (int j = 0; j < J; ++j) {
-    const int c = lane + 32 * j;
-    if (c < d) {
-      atomicAdd((unsigned long long*)&s.node_sum[c], (unsigned long long)accg[j]);
-      atomicAdd((unsigned long long*)&s.node_sum[d + c], (unsigned long long)acch[j]);
-    }
-  }
-  if (blockIdx.x == 0 && threadIdx.x < 32) {
     for (int c = lane; c < d; c += 32) {
+      const double pk = exp(pr[c] - mx) / sum;
+      const double g = pk - (double)y[i * d + c];
+      const double h = pk * (1.0 - pk);
+      q[i * V + c] = __double2int_rn(ldexp(g, kQShift));
+      q[i * V + d + c] = __double2int_rn(ldexp(h, kQShift + 2));
+    }
+  }
+  if (blockIdx.x == 0) {
+    for (int c = threadIdx.x; c < d; c += blockDim.x) {
       scales[c] = ldexpf(1.0f, -kQShift);
       scales[d + c] = ldexpf(1.0f, -kQShift - 2);
     }
+  }
+}
+
+// Exact column sums of q (root node totals).  block (32, 8): x = column within a group of 32.
+__global__ void k_qsum(gbdtmo_problem p, const int32_t* __restrict__ q, State s) {
+  __shared__ long long red[8][33];
+  const int V = channels(p);
+  for (int c0 = 0; c0 < V; c0 += 32) {
+    const int c = c0 + threadIdx.x;
+    long long acc = 0;
+    if (c < V)
+      for (int64_t i = blockIdx.x * 8 + threadIdx.y; i < p.n; i += (int64_t)gridDim.x * 8) acc += q[i * V + c];
+    red[threadIdx.y][threadIdx.x] = acc;
+    __syncthreads();
+    if (threadIdx.y == 0 && c < V) {
+      long long t = 0;
+      for (int r = 0; r < 8; ++r) t += red[r][threadIdx.x];
+      atomicAdd((unsigned long long*)&s.node_sum[c], (unsigned long long)t);
+    }
+    __syncthreads();
   }
 }
 
@@ -177,7 +168,6 @@ extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, cons
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
   GB_CHECK_ARG(y && pred && q && scales && state, "null pointer");
-  GB_CHECK_ARG(p->loss != GBDTMO_LOSS_SOFTMAX || p->d <= 256, "softmax supports d <= 256");
   State s = state_view(*p, state);
   const int sms = ctx->num_sms;
   GB_LAUNCH(k_tree_reset, sms, 256, 0, *p, s);
@@ -186,6 +176,7 @@ extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, cons
     GB_LAUNCH(k_mse_quantize, sms * 4, dim3(32, 8), 0, *p, y, pred, q, scales, s);
   } else {
     GB_LAUNCH(k_softmax_quantize, sms * 4, 256, 0, *p, y, pred, q, scales, s);
+    GB_LAUNCH(k_qsum, sms * 4, dim3(32, 8), 0, *p, q, s);
   }
   GB_LAUNCH(k_rows_init, sms * 4, 256, 0, *p, s);
   GB_LAUNCH(k_root_plan, 1, kPlanThreads, 0, *p, s, target_chunks_for(ctx, *p));

@@ -81,7 +81,13 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   __shared__ int sh_item;
   constexpr int RPI = 32 / K;                  // rows per warp instruction
   constexpr int G = K;                         // groups per 32-row batch
-  constexpr int SB = G < 8 ? G : 8;            // groups per q-prefetch sub-batch
+#ifndef GBDTMO_HIST_NOCOUNT
+#define GBDTMO_HIST_NOCOUNT 0      // (experiment only: drops the counts; results invalid)
+#endif
+#ifndef GBDTMO_HIST_SB
+#define GBDTMO_HIST_SB 8
+#endif
+  constexpr int SB = G < GBDTMO_HIST_SB ? G : GBDTMO_HIST_SB;   // groups per q-prefetch sub-batch
   constexpr int RS = KF * 2 * K;               // limb words per bin
   constexpr int NW = HistRow<KF>::NW, SW = HistRow<KF>::SW;
   const int V = channels(p), B = p.B, m = p.m;
@@ -155,7 +161,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       for (int i = 0; i < SW; ++i) sw[i] = 0;
       if (r >= 0) {
         shift_window<NW, SW>(w_cur, o, sw);
-        if (do_cnt) {
+        if (do_cnt && !GBDTMO_HIST_NOCOUNT) {
 #pragma unroll
           for (int j = 0; j < KF; ++j) {
             const uint32_t bin = byte_of<SW>(sw, j);
@@ -232,7 +238,6 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
-        const int j = e / B, b = e - j * B;
         const uint32_t nv = sm[limb_words + e];                    // counts[j][b], e = j * B + b
         if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }

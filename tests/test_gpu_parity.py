@@ -47,6 +47,7 @@ CASES = {
     "C3s": gen.WORKLOADS["C3"].scaled(n=100_000, m=24, T=3, D=6),
     "C4s": gen.WORKLOADS["C4"].scaled(n=20_000, m=20, T=2, D=4),
     "C5s": gen.WORKLOADS["C5"].scaled(n=50_000, m=70, T=2, D=5),
+    "S300s": gen.sweep(300, n=6_000, m=24, T=2, D=3),        # NEXT-2 class sweep, d = 300 softmax
 }
 
 
@@ -166,7 +167,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
 # ------------------------------------------------------------------- whole trees
 
 @pytest.mark.parametrize("case,sparse", [("C1", False), ("C2s", False), ("C2s", True), ("C3s", False),
-                                         ("C4s", False), ("C5s", False)])
+                                         ("C4s", False), ("C5s", False), ("S300s", False)])
 def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse):
     w = CASES[case]
     X, Y = _inputs(w)

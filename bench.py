@@ -218,8 +218,13 @@ def main():
 
     # ---- inputs in HBM (untimed): X shard generated on the device, binned by gbdtmo_bin
     t_setup = time.perf_counter()
-    Yh = host_targets(w)
-    Y = torch.from_numpy(Yh).to(dev)
+    # targets: computed once on rank 0's host and broadcast (every rank replicates y)
+    if rank == 0:
+        Y = torch.from_numpy(host_targets(w)).to(dev)
+    else:
+        Y = torch.empty((w.n, w.d), dtype=torch.float32, device=dev)
+    if group is not None:
+        dist.broadcast(Y, src=0, group=group)
     if w.classes_sweep:                 # features depend on the labels: generated on the host
         X = torch.from_numpy(gen.features_host(w, 0, w.n, f0, m_loc)).to(dev)
     else:
@@ -336,7 +341,9 @@ def main():
     del booster, ds
     torch.cuda.empty_cache()
     if not a.no_e2e:
-        out["e2e"] = e2e_run(w, a, rank, world, local, dev, group, f0, f1)
+        Yhost = Y.cpu().pin_memory()
+        del Y
+        out["e2e"] = e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yhost)
 
     if group is not None:
         dist.barrier()
@@ -352,7 +359,7 @@ def main():
     return 0
 
 
-def e2e_run(w, a, rank, world, local, dev, group, f0, f1):
+def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh):
     """train(): pinned host X shard + y -> H2D -> gbdtmo_bin -> K trees -> D2H of yhat and the trees."""
     import torch
     import torch.distributed as dist
@@ -362,7 +369,6 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1):
     Xh = torch.empty((w.n, m_loc), dtype=torch.float32, pin_memory=True)
     Xh.numpy()[:] = gen.features_host(w, 0, w.n, f0, m_loc) if w.classes_sweep else \
         gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, f0, m_loc, w.m, out=Xh.numpy())
-    Yh = torch.from_numpy(host_targets(w)).pin_memory()
     ctx = pkg.Context(local)
     params = pkg.Params(loss=w.loss, T=a.steps, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
                         min_node=w.min_node)

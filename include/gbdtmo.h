@@ -96,6 +96,14 @@ gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out /* host */);
 gbdtmo_status gbdtmo_destroy(gbdtmo_ctx ctx);
 gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx ctx, void* cuda_stream /* cudaStream_t */);
 const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
+/* Context options (apply to subsequent calls on the context):
+ *   GBDTMO_OPT_GMEM_MAX_ROWS: histogram variant selection — BUILD nodes with at most this many
+ *     rows use the global-atomic variant (one REDG per (row, feature, channel) into the node's
+ *     histogram) instead of the shared-memory privatised variant;
+ *     0 (default) = shared memory for every node.  The threshold comes from measurement
+ *     (tools/calibrate_hist.py). */
+enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1 };
+gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Number of kernels this context has launched so far (for launch accounting). */
 int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
 

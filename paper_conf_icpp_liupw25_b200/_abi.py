@@ -25,7 +25,9 @@ SYMBOLS = (
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
+    "gbdtmo_set_option",
 )
+OPT_GMEM_MAX_ROWS = 1
 
 
 class GbdtmoError(RuntimeError):
@@ -61,6 +63,7 @@ def lib():
             "gbdtmo_destroy": ([P], C.c_int),
             "gbdtmo_set_stream": ([P, P], C.c_int),
             "gbdtmo_last_error": ([P], C.c_char_p),
+            "gbdtmo_set_option": ([P, i32, i64], C.c_int),
             "gbdtmo_launch_count": ([P], i64),
             "gbdtmo_bins_bytes": ([i64, i64], sz),
             "gbdtmo_bin_workspace_bytes": ([i64, i32, i32], sz),
@@ -124,6 +127,9 @@ class Context:
     # lifecycle -------------------------------------------------------------
     def gbdtmo_set_stream(self, stream_handle: int):
         self._check(lib().gbdtmo_set_stream(self._h, C.c_void_p(stream_handle)), "gbdtmo_set_stream")
+
+    def gbdtmo_set_option(self, option: int, value: int):
+        self._check(lib().gbdtmo_set_option(self._h, option, value), "gbdtmo_set_option")
 
     def gbdtmo_launch_count(self) -> int:
         return int(lib().gbdtmo_launch_count(self._h))

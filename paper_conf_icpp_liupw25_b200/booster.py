@@ -34,6 +34,29 @@ class Params:
     min_node: int = 20
 
 
+# Measured histogram-variant table (tools/calibrate_hist.py -> profiles/hist_variant_table.json):
+# largest node size (rows) for which the global-atomic variant beat the shared-memory variant,
+# per channel count V.  Empty until calibrated: shared memory everywhere.
+_VARIANT_TABLE = None
+
+
+def variant_threshold(V: int, m: int) -> int:
+    global _VARIANT_TABLE
+    if _VARIANT_TABLE is None:
+        import json
+        import os
+        path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "hist_variant_table.json")
+        try:
+            _VARIANT_TABLE = json.load(open(path))
+        except (OSError, ValueError):
+            _VARIANT_TABLE = {}
+    entries = _VARIANT_TABLE.get("entries", [])
+    if not entries:
+        return 0
+    e = min(entries, key=lambda e: abs(e["V"] - V))      # nearest measured channel count
+    return int(e["gmem_max_rows"])
+
+
 def _align(x, a):
     return (x + a - 1) // a * a
 
@@ -81,8 +104,12 @@ class Booster:
 
     def __init__(self, ctx: Context, ds: Dataset, y: torch.Tensor, params: Params,
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
-                 sparse_default: bool = False):
+                 sparse_default: bool = False, gmem_max_rows: Optional[int] = None):
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
+        # histogram variant selection: nodes with <= gmem_max_rows
+        # rows use the global-atomic variant; None = the measured table for this channel count
+        self.gmem_max_rows = variant_threshold(y.shape[1] * (2 if params.loss == LOSS_SOFTMAX else 1),
+                                               ds.m) if gmem_max_rows is None else int(gmem_max_rows)
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
@@ -147,6 +174,7 @@ class Booster:
     def _tree(self, time_hist: bool = False):
         ctx, p = self.ctx, self.p
         ctx.gbdtmo_set_stream(torch.cuda.current_stream(self.device).cuda_stream)
+        ctx.gbdtmo_set_option(_abi.OPT_GMEM_MAX_ROWS, self.gmem_max_rows)
         ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state)
         for lvl in range(self.params.D):
             self._level(lvl, time_hist)

@@ -41,6 +41,15 @@ extern "C" gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx c, void* stream) {
   return GBDTMO_OK;
 }
 
+extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t value) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  switch (option) {
+    case GBDTMO_OPT_GMEM_MAX_ROWS: ctx->gmem_max_rows = value; return GBDTMO_OK;
+    default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;
+  }
+}
+
 extern "C" const char* gbdtmo_last_error(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
   return ctx ? ctx->err.c_str() : "null context";

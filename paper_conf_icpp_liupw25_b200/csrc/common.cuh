@@ -20,6 +20,7 @@ struct Ctx {
   int num_sms = 148;
   int max_smem_optin = 227 * 1024;
   int64_t launches = 0;
+  int64_t gmem_max_rows = 0;   // GBDTMO_OPT_GMEM_MAX_ROWS: BUILD nodes with <= rows use the global-atomic variant
   std::string err;
 };
 
@@ -54,7 +55,9 @@ constexpr int kHistSmemBudget = 218 * 1024;   // limbs + counts + per-warp row s
 constexpr int kHistWarps = kHistThreads / 32;
 constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte bin window)
 
-enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2 };
+// MODE_BUILD1: built by exactly one work item per tile -> the flush stores instead of adding, and
+// the slot needs no zeroing (saves 2 passes over the node's histogram in HBM).
+enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2, MODE_BUILD1 = 3 };
 
 __host__ __device__ inline int channels(const gbdtmo_problem& p) {
   return p.loss == GBDTMO_LOSS_SOFTMAX ? 2 * p.d : p.d;
@@ -105,7 +108,7 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
 struct StateLayout {
   size_t rows0, rows1, nid;
   size_t node_begin, node_end, node_state, node_mode, node_feat, node_bin, node_gain, node_nleft, node_sum;
-  size_t chunks, misc, scale_max, tile_cnt, lpart;
+  size_t chunks, gnodes, misc, scale_max, tile_cnt, lpart;
   size_t total;
 };
 
@@ -129,6 +132,7 @@ __host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
   L.node_nleft = take(8 * NH);
   L.node_sum = take(8 * NH * (V + 1));
   L.chunks = take(16 * (size_t)max_chunks(p));
+  L.gnodes = take(16 * (size_t)(max_level_nodes(p) + 1));
   L.misc = take(64);
   L.scale_max = take(8 * V);
   L.tile_cnt = take(4 * ((size_t)part_tiles(p) + 1));
@@ -138,7 +142,7 @@ __host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
 }
 
 // misc words
-enum { MISC_CHUNK_COUNT = 0, MISC_WORK_COUNTER = 1, MISC_CHUNK_ROWS = 2 };
+enum { MISC_CHUNK_COUNT = 0, MISC_WORK_COUNTER = 1, MISC_CHUNK_ROWS = 2, MISC_GNODE_COUNT = 3, MISC_GNODE_ROWS = 4 };
 
 struct State {
   int32_t *rows0, *rows1, *nid;
@@ -147,6 +151,7 @@ struct State {
   int64_t* node_nleft;
   int64_t* node_sum;  // [NH][V+1]: V channel sums of q, then the row count
   int4* chunks;       // (slot, begin, end, unused)
+  int4* gnodes;       // global-atomic variant nodes: (slot, begin, end, row prefix)
   int32_t* misc;
   unsigned long long* scale_max;   // bits of max_i |g_ic| (fp64, non-negative)
   int32_t* tile_cnt;
@@ -170,6 +175,7 @@ __host__ __device__ inline State state_view(const gbdtmo_problem& p, void* base)
   s.node_nleft = (int64_t*)(b + L.node_nleft);
   s.node_sum = (int64_t*)(b + L.node_sum);
   s.chunks = (int4*)(b + L.chunks);
+  s.gnodes = (int4*)(b + L.gnodes);
   s.misc = (int32_t*)(b + L.misc);
   s.scale_max = (unsigned long long*)(b + L.scale_max);
   s.tile_cnt = (int32_t*)(b + L.tile_cnt);

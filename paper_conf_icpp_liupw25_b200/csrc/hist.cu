@@ -221,8 +221,10 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     }
     __syncthreads();
 
-    // flush: exact int64 = hi * 2^16 + lo into the node histogram (global REDG.ADD.64)
+    // flush: exact int64 = hi * 2^16 + lo into the node histogram (global REDG.ADD.64, or plain
+    // stores of every entry when this item is the node's only writer: no zeroing, no read-back)
     const int64_t slot = ch.x;
+    const bool sole = ch.w != 0;
     const int64_t gbase = (slot * m + f0) * (int64_t)B;        // (slot, f0, bin 0)
     const int total = kk * B * K;
     for (int e = threadIdx.x; e < total; e += blockDim.x) {
@@ -232,17 +234,64 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       const uint32_t* rowp = sm + b * RS + j * 2 * K;
       const uint32_t los = rowp[cc], his = rowp[K + cc];
       const long long v = (long long)(int32_t)his * 65536LL + (long long)los;
-      if (v != 0)   // channel-major node histogram: [f][c][b]
-        atomicAdd(reinterpret_cast<unsigned long long*>(&hist[((slot * m + f0 + j) * V + c0 + cc) * B + b]),
-                  (unsigned long long)v);
+      int64_t* dst = &hist[((slot * m + f0 + j) * V + c0 + cc) * B + b];   // channel-major [f][c][b]
+      if (sole) *dst = v;
+      else if (v != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst), (unsigned long long)v);
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
         const uint32_t nv = sm[limb_words + e];                    // counts[j][b], e = j * B + b
-        if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
+        if (sole) cnt[gbase + e] = (int32_t)nv;
+        else if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }
     }
     __syncthreads();
+  }
+}
+
+// Global-atomic variant (the paper's "global memory approach"; for small nodes,
+// where the shared-memory variant's per-item zero/flush of ~200 KB tiles dominates): one warp
+// per row of the level's small BUILD nodes, lanes over features, one REDG.ADD.64 per
+// (row, feature, channel) straight into the node's (zeroed) int64 histogram.
+template <bool SKIP>
+__global__ void __launch_bounds__(256)
+k_hist_gmem(gbdtmo_problem p, const uint8_t* __restrict__ bins, const int32_t* __restrict__ dflt,
+            const int32_t* __restrict__ q, const int32_t* __restrict__ rows, int use_rows, State s,
+            int64_t* __restrict__ hist, int32_t* __restrict__ cnt) {
+  __shared__ int4 gn[512];
+  const int ng = s.misc[MISC_GNODE_COUNT];
+  const int total = s.misc[MISC_GNODE_ROWS];
+  if (ng == 0) return;
+  const int V = channels(p), B = p.B, m = p.m;
+  const int lane = threadIdx.x & 31;
+  const int64_t wid = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int base = 0; base < ng; base += 512) {        // node lists longer than 512: in slices
+    const int cnt_here = min(512, ng - base);
+    __syncthreads();
+    for (int i = threadIdx.x; i < cnt_here; i += blockDim.x) gn[i] = s.gnodes[base + i];
+    __syncthreads();
+    const int r_lo = gn[0].w, r_hi = (base + cnt_here < ng) ? s.gnodes[base + cnt_here].w : total;
+    for (int64_t ri = r_lo + wid; ri < r_hi; ri += nwarps) {
+      int lo = 0, hi = cnt_here - 1;                  // last node with prefix <= ri
+      while (lo < hi) { const int mid = (lo + hi + 1) >> 1; if (gn[mid].w <= ri) lo = mid; else hi = mid - 1; }
+      const int4 nd = gn[lo];
+      const int pos = nd.y + (int)(ri - nd.w);
+      const int r = use_rows ? __ldg(&rows[pos]) : pos;
+      const uint8_t* br = bins + (int64_t)r * p.ld_bins;
+      const int32_t* qr = q + (int64_t)r * V;
+      const int64_t sbase = (int64_t)nd.x * m;
+      for (int f = lane; f < m; f += 32) {
+        const int b = br[f];
+        if (SKIP && b == __ldg(&dflt[f])) continue;
+        atomicAdd(&cnt[(sbase + f) * B + b], 1);
+        int64_t* hb = hist + (sbase + f) * V * B + b;
+        for (int c = 0; c < V; ++c) {
+          const int v = __ldg(&qr[c]);
+          if (v) atomicAdd(reinterpret_cast<unsigned long long*>(hb + (int64_t)c * B), (unsigned long long)(long long)v);
+        }
+      }
+    }
   }
 }
 
@@ -328,9 +377,14 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
   GB_LAUNCH(k_zero_build, dim3(gx, (unsigned)LN), 256, 0, *p, level, s, hist, cnt);
   const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
   const int use_rows = level > 0;
+  gbdtmo_status st;
   switch (hc.K) {
-    case 4: return launch_hist<4>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 8: return launch_hist<8>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    default: return launch_hist<16>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 4: st = launch_hist<4>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
+    case 8: st = launch_hist<8>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
+    default: st = launch_hist<16>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
   }
+  if (st != GBDTMO_OK || ctx->gmem_max_rows <= 0) return st;
+  if (dflt) GB_LAUNCH(k_hist_gmem<true>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  else GB_LAUNCH(k_hist_gmem<false>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  return GBDTMO_OK;
 }

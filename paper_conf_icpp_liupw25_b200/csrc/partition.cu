@@ -11,7 +11,8 @@ namespace gbdtmo {
 
 // Apply the merged records: decisions for the level's nodes, child nodes, next-level plan.
 __global__ void __launch_bounds__(kPlanThreads)
-k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ xchg, int target_chunks) {
+k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ xchg, int target_chunks,
+                int64_t gmem_max_rows) {
   const int64_t LN = int64_t(1) << level, first = LN - 1;
   const int V = channels(p);
   const int64_t RW = rec_words(p);
@@ -54,7 +55,7 @@ k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict_
     s.node_mode[hg] = mg;
   }
   __syncthreads();
-  plan_level_chunks(p, s, level + 1, target_chunks);
+  plan_level_chunks(p, s, level + 1, target_chunks, gmem_max_rows);
 }
 
 __device__ __forceinline__ bool bitmap_bit(const int64_t* __restrict__ bm, int32_t r) {
@@ -209,7 +210,8 @@ extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p,
   const int32_t* rows_in = (level & 1) ? s.rows1 : s.rows0;
   int32_t* rows_out = (level & 1) ? s.rows0 : s.rows1;
   const int64_t ntiles = part_tiles(*p);
-  GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p));
+  GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p),
+            ctx->gmem_max_rows);
   GB_LAUNCH(k_part_count, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, bm);
   GB_LAUNCH(k_part_scan, 1, kPartThreads, 0, ntiles, s);
   GB_LAUNCH(k_part_scatter, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, rows_out, bm);

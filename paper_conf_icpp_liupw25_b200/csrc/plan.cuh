@@ -39,16 +39,17 @@ __device__ inline int block_excl_scan_256(int v, int* total) {
 // Write the build chunks of `level` into s.chunks: every node of the level with mode BUILD
 // is cut into pieces of R rows, R = clamp(ceil(build_rows / target_chunks), kChunkMin, kChunkMax).
 __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s, int level,
-                                         int target_chunks) {
+                                         int target_chunks, int64_t gmem_max_rows) {
   const int64_t LN = int64_t(1) << level, first = LN - 1;
   __shared__ long long sh_rows;
   __shared__ int sh_R, sh_base;
   if (threadIdx.x == 0) { sh_rows = 0; sh_base = 0; }
   __syncthreads();
   long long my = 0;
+  auto is_gmem = [&](int64_t h) { return (int64_t)(s.node_end[h] - s.node_begin[h]) <= gmem_max_rows; };
   for (int64_t i = threadIdx.x; i < LN; i += blockDim.x) {
     int64_t h = first + i;
-    if (s.node_mode[h] == MODE_BUILD) my += s.node_end[h] - s.node_begin[h];
+    if (s.node_mode[h] == MODE_BUILD && !is_gmem(h)) my += s.node_end[h] - s.node_begin[h];
   }
   atomicAdd((unsigned long long*)&sh_rows, (unsigned long long)my);
   __syncthreads();
@@ -66,7 +67,7 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     int nchunk = 0, b = 0, e = 0;
     if (i < LN) {
       int64_t h = first + i;
-      if (s.node_mode[h] == MODE_BUILD) {
+      if (s.node_mode[h] == MODE_BUILD && !is_gmem(h)) {
         b = s.node_begin[h]; e = s.node_end[h];
         nchunk = (e - b + R - 1) / R;
       }
@@ -76,8 +77,9 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     for (int c = 0; c < nchunk; ++c) {
       int cb = b + c * R;
       int ce = cb + R < e ? cb + R : e;
-      s.chunks[off + c] = make_int4((int)i, cb, ce, 0);
+      s.chunks[off + c] = make_int4((int)i, cb, ce, nchunk == 1 ? 1 : 0);   // w = 1: sole writer
     }
+    if (nchunk == 1) s.node_mode[first + i] = MODE_BUILD1;
     __syncthreads();
     if (threadIdx.x == 0) sh_base += total;
     __syncthreads();
@@ -86,6 +88,30 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     s.misc[MISC_CHUNK_COUNT] = sh_base;
     s.misc[MISC_WORK_COUNTER] = 0;
     s.misc[MISC_CHUNK_ROWS] = R;
+  }
+  __syncthreads();
+  // small BUILD nodes -> the global-atomic variant's list, with an exclusive row prefix
+  __shared__ int sh_gn, sh_gr;
+  if (threadIdx.x == 0) { sh_gn = 0; sh_gr = 0; }
+  __syncthreads();
+  for (int64_t i0 = 0; i0 < LN; i0 += blockDim.x) {
+    const int64_t i = i0 + threadIdx.x;
+    int take = 0, rows = 0, b = 0, e = 0;
+    if (i < LN) {
+      const int64_t h = first + i;
+      if (s.node_mode[h] == MODE_BUILD && is_gmem(h)) { take = 1; b = s.node_begin[h]; e = s.node_end[h]; rows = e - b; }
+    }
+    int tn, tr;
+    const int on = block_excl_scan_256(take, &tn);
+    const int orow = block_excl_scan_256(rows, &tr);
+    if (take) s.gnodes[sh_gn + on] = make_int4((int)i, b, e, sh_gr + orow);
+    __syncthreads();
+    if (threadIdx.x == 0) { sh_gn += tn; sh_gr += tr; }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    s.misc[MISC_GNODE_COUNT] = sh_gn;
+    s.misc[MISC_GNODE_ROWS] = sh_gr;
   }
 }
 

@@ -166,16 +166,17 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------- whole trees
 
-@pytest.mark.parametrize("case,sparse", [("C1", False), ("C2s", False), ("C2s", True), ("C3s", False),
-                                         ("C4s", False), ("C5s", False), ("S300s", False)])
-def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse):
+@pytest.mark.parametrize("case,sparse,gmem", [("C1", False, 0), ("C2s", False, 0), ("C2s", True, 0), ("C3s", False, 0),
+                                              ("C4s", False, 0), ("C5s", False, 0), ("S300s", False, 0),
+                                              ("C3s", False, 1 << 30), ("C2s", True, 3000), ("C5s", False, 5000)])
+def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem):
     w = CASES[case]
     X, Y = _inputs(w)
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
     ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
                     lr=w.lr, min_node=w.min_node)
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse, gmem_max_rows=gmem)
     assert (b.dflt is not None) == (sparse and w.index == 2)     # only the MNIST-shaped data has dominant bins
     b.fit()
     torch.cuda.synchronize()

@@ -1,0 +1,69 @@
+"""Measure the histogram-variant crossover (shared-memory privatised vs global atomics) per
+channel count and write paper_conf_icpp_liupw25_b200/hist_variant_table.json, the table the
+Booster's per-node variant selection reads.
+
+  python tools/calibrate_hist.py            (on a B200, ~2 minutes)
+
+For each workload shape, trains 2 warm-up + 3 timed trees at every candidate threshold
+(BUILD nodes with <= threshold rows use the global-atomic variant) and keeps the fastest.
+"""
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import paper_conf_icpp_liupw25_b200 as pkg  # noqa: E402
+from gen import gen  # noqa: E402
+
+CANDIDATES = [0, 256, 512, 1024, 2048, 4096, 8192, 16384]
+
+
+def time_trees(ctx, ds, Y, w, thr, warm=2, timed=3):
+    P = pkg.Params(loss=w.loss, T=warm + timed, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
+                   min_node=w.min_node)
+    b = pkg.Booster(ctx, ds, Y, P, keep_model=False, gmem_max_rows=thr)
+    for _ in range(warm):
+        b.step()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(timed):
+        b.step()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / timed
+
+
+def main():
+    shapes = [gen.WORKLOADS["C2"], gen.WORKLOADS["C3"], gen.sweep(5), gen.sweep(100),
+              gen.WORKLOADS["C5"].scaled(n=500_000, m=1024)]
+    ctx = pkg.Context(0)
+    entries = []
+    for w in shapes:
+        X = torch.from_numpy(gen.features_host(w)).cuda()
+        ds = pkg.bin_features(ctx, X, w.B)
+        del X
+        Y = torch.from_numpy(gen.targets_host(w)).cuda()
+        V = w.d * (2 if w.loss == gen.LOSS_SOFTMAX else 1)
+        res = {c: time_trees(ctx, ds, Y, w, c) for c in CANDIDATES}
+        best = min(res, key=res.get)
+        entries.append({"workload": w.name, "V": V, "m": w.m, "n": w.n, "gmem_max_rows": best,
+                        "ms_per_tree": {str(k): round(v, 4) for k, v in res.items()}})
+        print(json.dumps(entries[-1]), flush=True)
+        del ds, Y
+        torch.cuda.empty_cache()
+    out = {"measured": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
+           "device": torch.cuda.get_device_name(0), "candidates": CANDIDATES, "entries": entries}
+    path = os.path.join(ROOT, "paper_conf_icpp_liupw25_b200", "hist_variant_table.json")
+    json.dump(out, open(path, "w"), indent=1)
+    os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+    json.dump(out, open(os.path.join(ROOT, "gpurun_out", "hist_variant_table.json"), "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()

@@ -101,8 +101,12 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *     rows use the global-atomic variant (one REDG per (row, feature, channel) into the node's
  *     histogram) instead of the shared-memory privatised variant;
  *     0 (default) = shared memory for every node.  The threshold comes from measurement
- *     (tools/calibrate_hist.py). */
-enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1 };
+ *     (tools/calibrate_hist.py).
+ *   GBDTMO_OPT_SMALL_MAX_ROWS: fused small-node path — when both children of a split have at most
+ *     this many rows they are marked SMALL: built from their rows and searched in shared memory by
+ *     gbdtmo_search_small, never materialised and not derived by subtraction (reading R27);
+ *     0 (default) = off.  Requires d <= 32 and a feature tile that fits shared memory. */
+enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2 };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Number of kernels this context has launched so far (for launch accounting). */
 int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
@@ -200,6 +204,15 @@ gbdtmo_status gbdtmo_find_split(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t
                                 const int64_t* parent_hist, const int32_t* parent_cnt,
                                 uint64_t* keys);
 
+/* (a)3 + (a)5 fused for small nodes: for every node of `level` marked SMALL (see
+ * GBDTMO_OPT_SMALL_MAX_ROWS) build its histograms from its rows in shared memory and evaluate
+ * Eq. (3) in place, max-reducing the packed keys into keys[slot] (same key and tie rule as
+ * gbdtmo_find_split); nothing is written to the global histograms.  Call after
+ * gbdtmo_find_split (which zeroes keys) and before the key exchange.  No-op when the option is 0. */
+gbdtmo_status gbdtmo_search_small(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                  const uint8_t* bins, const int32_t* q, const int32_t* nbins,
+                                  const float* scales, void* state, uint64_t* keys);
+
 /* ------------------------------------------------------------ (a)6 exchange */
 
 /* Split records of `level`, written by the process that owns each winning feature
@@ -213,9 +226,11 @@ gbdtmo_status gbdtmo_find_split(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t
  *                            splitting node of this level and goes left (bin <= b).
  * keys: this level's keys after the (optional) MAX all-reduce; scales from gbdtmo_grad;
  * hist / cnt / parent_hist / parent_cnt as for gbdtmo_find_split (a derived winner's sums are
- * parent - sibling).  Every xchg word is written. */
+ * parent - sibling); q from gbdtmo_grad (the left sums of a SMALL winner are summed from its
+ * rows).  Every xchg word is written. */
 gbdtmo_status gbdtmo_split_record(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
-                                  const uint8_t* bins, const int32_t* dflt, const float* scales, void* state,
+                                  const uint8_t* bins, const int32_t* dflt, const int32_t* q,
+                                  const float* scales, void* state,
                                   const int64_t* hist, const int32_t* cnt,
                                   const int64_t* parent_hist, const int32_t* parent_cnt,
                                   const uint64_t* keys, int64_t* xchg);

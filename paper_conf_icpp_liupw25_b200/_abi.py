@@ -25,9 +25,9 @@ SYMBOLS = (
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
-    "gbdtmo_set_option",
+    "gbdtmo_set_option", "gbdtmo_search_small",
 )
-OPT_GMEM_MAX_ROWS = 1
+OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS = 1, 2
 
 
 class GbdtmoError(RuntimeError):
@@ -75,7 +75,8 @@ def lib():
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
-            "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_search_small": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
             "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
@@ -186,10 +187,14 @@ class Context:
                                             _ptr(state), _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
                                             _ptr(keys)), "gbdtmo_find_split")
 
-    def gbdtmo_split_record(self, p, level, bins, dflt, scales, state, hist, cnt, parent_hist, parent_cnt, keys,
+    def gbdtmo_search_small(self, p, level, bins, q, nbins, scales, state, keys):
+        self._check(lib().gbdtmo_search_small(self._h, C.byref(p), level, _ptr(bins), _ptr(q), _ptr(nbins),
+                                              _ptr(scales), _ptr(state), _ptr(keys)), "gbdtmo_search_small")
+
+    def gbdtmo_split_record(self, p, level, bins, dflt, q, scales, state, hist, cnt, parent_hist, parent_cnt, keys,
                             xchg):
-        self._check(lib().gbdtmo_split_record(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(scales),
-                                              _ptr(state),
+        self._check(lib().gbdtmo_split_record(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(q),
+                                              _ptr(scales), _ptr(state),
                                               _ptr(hist), _ptr(cnt), _ptr(parent_hist), _ptr(parent_cnt),
                                               _ptr(keys), _ptr(xchg)), "gbdtmo_split_record")
 

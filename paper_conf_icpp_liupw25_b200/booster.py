@@ -40,7 +40,7 @@ class Params:
 _VARIANT_TABLE = None
 
 
-def variant_threshold(V: int, m: int) -> int:
+def variant_threshold(V: int, m: int, key: str = "gmem_max_rows") -> int:
     global _VARIANT_TABLE
     if _VARIANT_TABLE is None:
         import json
@@ -54,7 +54,7 @@ def variant_threshold(V: int, m: int) -> int:
     if not entries:
         return 0
     e = min(entries, key=lambda e: abs(e["V"] - V))      # nearest measured channel count
-    return int(e["gmem_max_rows"])
+    return int(e.get(key, 0))
 
 
 def _align(x, a):
@@ -104,12 +104,15 @@ class Booster:
 
     def __init__(self, ctx: Context, ds: Dataset, y: torch.Tensor, params: Params,
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
-                 sparse_default: bool = False, gmem_max_rows: Optional[int] = None):
+                 sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
+                 small_max_rows: Optional[int] = None):
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
         # histogram variant selection: nodes with <= gmem_max_rows
         # rows use the global-atomic variant; None = the measured table for this channel count
-        self.gmem_max_rows = variant_threshold(y.shape[1] * (2 if params.loss == LOSS_SOFTMAX else 1),
-                                               ds.m) if gmem_max_rows is None else int(gmem_max_rows)
+        V = y.shape[1] * (2 if params.loss == LOSS_SOFTMAX else 1)
+        self.gmem_max_rows = variant_threshold(V, ds.m) if gmem_max_rows is None else int(gmem_max_rows)
+        self.small_max_rows = variant_threshold(V, ds.m, "small_max_rows") if small_max_rows is None \
+            else int(small_max_rows)
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
@@ -163,18 +166,27 @@ class Booster:
             self.hist_events.append((e0, e1))
         ctx.gbdtmo_find_split(p, lvl, self.ds.nbins, self.dflt, self.scales, self.state, self.hist[cur], self.cnt[cur],
                               ph, pc, self.keys)
+        if self.small_max_rows > 0:
+            ctx.gbdtmo_search_small(p, lvl, self.ds.bins, self.q, self.ds.nbins, self.scales, self.state, self.keys)
         if self.group is not None:
             parallel.exchange_keys(self.keys[: 1 << lvl], self.group)
-        ctx.gbdtmo_split_record(p, lvl, self.ds.bins, self.dflt, self.scales, self.state, self.hist[cur], self.cnt[cur],
+        ctx.gbdtmo_split_record(p, lvl, self.ds.bins, self.dflt, self.q, self.scales, self.state, self.hist[cur],
+                                self.cnt[cur],
                                 ph, pc, self.keys, self.xchg)
         if self.group is not None:
             parallel.exchange_records(self.xchg, self.group)
         ctx.gbdtmo_partition(p, lvl, self.state, self.xchg)
 
-    def _tree(self, time_hist: bool = False):
-        ctx, p = self.ctx, self.p
+    def _apply_options(self):
+        """Context state for this booster's calls: stream and histogram-variant thresholds."""
+        ctx = self.ctx
         ctx.gbdtmo_set_stream(torch.cuda.current_stream(self.device).cuda_stream)
         ctx.gbdtmo_set_option(_abi.OPT_GMEM_MAX_ROWS, self.gmem_max_rows)
+        ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
+
+    def _tree(self, time_hist: bool = False):
+        ctx, p = self.ctx, self.p
+        self._apply_options()
         ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state)
         for lvl in range(self.params.D):
             self._level(lvl, time_hist)

@@ -46,6 +46,7 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
   if (!ctx) return GBDTMO_EINVAL;
   switch (option) {
     case GBDTMO_OPT_GMEM_MAX_ROWS: ctx->gmem_max_rows = value; return GBDTMO_OK;
+    case GBDTMO_OPT_SMALL_MAX_ROWS: ctx->small_max_rows = value; return GBDTMO_OK;
     default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;
   }
 }

@@ -21,6 +21,7 @@ struct Ctx {
   int max_smem_optin = 227 * 1024;
   int64_t launches = 0;
   int64_t gmem_max_rows = 0;   // GBDTMO_OPT_GMEM_MAX_ROWS: BUILD nodes with <= rows use the global-atomic variant
+  int64_t small_max_rows = 0;  // GBDTMO_OPT_SMALL_MAX_ROWS: nodes whose parent's children both fit -> fused path
   std::string err;
 };
 
@@ -57,7 +58,13 @@ constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte b
 
 // MODE_BUILD1: built by exactly one work item per tile -> the flush stores instead of adding, and
 // the slot needs no zeroing (saves 2 passes over the node's histogram in HBM).
-enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2, MODE_BUILD1 = 3 };
+// MODE_SMALL: built from its rows and searched in shared memory (small.cu), never materialised.
+enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2, MODE_BUILD1 = 3, MODE_SMALL = 4 };
+
+// Packed split key: larger gain wins, ties -> smallest (f_global * B + b).
+__device__ __forceinline__ uint64_t pack_split_key(double gain, int64_t fb) {
+  return ((uint64_t)__double_as_longlong(gain) & ~0xFFFFFFull) | (uint64_t)(0xFFFFFF - fb);
+}
 
 __host__ __device__ inline int channels(const gbdtmo_problem& p) {
   return p.loss == GBDTMO_LOSS_SOFTMAX ? 2 * p.d : p.d;
@@ -108,7 +115,7 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
 struct StateLayout {
   size_t rows0, rows1, nid;
   size_t node_begin, node_end, node_state, node_mode, node_feat, node_bin, node_gain, node_nleft, node_sum;
-  size_t chunks, gnodes, misc, scale_max, tile_cnt, lpart;
+  size_t chunks, gnodes, snodes, misc, scale_max, tile_cnt, lpart;
   size_t total;
 };
 
@@ -133,6 +140,7 @@ __host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
   L.node_sum = take(8 * NH * (V + 1));
   L.chunks = take(16 * (size_t)max_chunks(p));
   L.gnodes = take(16 * (size_t)(max_level_nodes(p) + 1));
+  L.snodes = take(16 * (size_t)(max_level_nodes(p) + 1));
   L.misc = take(64);
   L.scale_max = take(8 * V);
   L.tile_cnt = take(4 * ((size_t)part_tiles(p) + 1));
@@ -142,7 +150,8 @@ __host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
 }
 
 // misc words
-enum { MISC_CHUNK_COUNT = 0, MISC_WORK_COUNTER = 1, MISC_CHUNK_ROWS = 2, MISC_GNODE_COUNT = 3, MISC_GNODE_ROWS = 4 };
+enum { MISC_CHUNK_COUNT = 0, MISC_WORK_COUNTER = 1, MISC_CHUNK_ROWS = 2, MISC_GNODE_COUNT = 3, MISC_GNODE_ROWS = 4,
+       MISC_SNODE_COUNT = 5, MISC_SWORK_COUNTER = 6 };
 
 struct State {
   int32_t *rows0, *rows1, *nid;
@@ -152,6 +161,7 @@ struct State {
   int64_t* node_sum;  // [NH][V+1]: V channel sums of q, then the row count
   int4* chunks;       // (slot, begin, end, unused)
   int4* gnodes;       // global-atomic variant nodes: (slot, begin, end, row prefix)
+  int4* snodes;       // fused small-node path: (slot, begin, end, unused)
   int32_t* misc;
   unsigned long long* scale_max;   // bits of max_i |g_ic| (fp64, non-negative)
   int32_t* tile_cnt;
@@ -176,6 +186,7 @@ __host__ __device__ inline State state_view(const gbdtmo_problem& p, void* base)
   s.node_sum = (int64_t*)(b + L.node_sum);
   s.chunks = (int4*)(b + L.chunks);
   s.gnodes = (int4*)(b + L.gnodes);
+  s.snodes = (int4*)(b + L.snodes);
   s.misc = (int32_t*)(b + L.misc);
   s.scale_max = (unsigned long long*)(b + L.scale_max);
   s.tile_cnt = (int32_t*)(b + L.tile_cnt);
@@ -204,6 +215,11 @@ inline const char* check_problem(const gbdtmo_problem* p) {
 
 // Histogram work items wanted per level -> chunks per build level (grad.cu).
 int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p);
+// Whether the fused small-node path fits this problem (small.cu); the effective threshold.
+bool small_supported(const gbdtmo_problem& p);
+inline int64_t small_rows(const Ctx* ctx, const gbdtmo_problem& p) {
+  return (ctx->small_max_rows > 0 && small_supported(p)) ? ctx->small_max_rows : 0;
+}
 
 // Launch helpers: count kernels and check errors.
 #define GB_LAUNCH(kernel, grid, block, smem, ...)                 \

@@ -135,7 +135,8 @@ __global__ void k_rows_init(gbdtmo_problem p, State s) {
   }
 }
 
-__global__ void k_root_plan(gbdtmo_problem p, State s, int target_chunks, int64_t gmem_max_rows) {
+__global__ void k_root_plan(gbdtmo_problem p, State s, int target_chunks, int64_t gmem_max_rows,
+                            int64_t small_max_rows) {
   const int64_t V = channels(p);
   if (threadIdx.x == 0) {
     s.node_begin[0] = 0;
@@ -143,7 +144,7 @@ __global__ void k_root_plan(gbdtmo_problem p, State s, int target_chunks, int64_
     s.node_sum[V] = p.n;
     bool active = p.D >= 1 && p.n >= 2 * (int64_t)p.min_node;
     s.node_state[0] = active ? GBDTMO_NODE_ACTIVE : GBDTMO_NODE_LEAF;
-    s.node_mode[0] = active ? MODE_BUILD : MODE_NONE;
+    s.node_mode[0] = active ? (p.n <= small_max_rows ? MODE_SMALL : MODE_BUILD) : MODE_NONE;
   }
   __syncthreads();
   plan_level_chunks(p, s, 0, target_chunks, gmem_max_rows);
@@ -179,6 +180,7 @@ extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, cons
     GB_LAUNCH(k_qsum, sms * 4, dim3(32, 8), 0, *p, q, s);
   }
   GB_LAUNCH(k_rows_init, sms * 4, 256, 0, *p, s);
-  GB_LAUNCH(k_root_plan, 1, kPlanThreads, 0, *p, s, target_chunks_for(ctx, *p), ctx->gmem_max_rows);
+  GB_LAUNCH(k_root_plan, 1, kPlanThreads, 0, *p, s, target_chunks_for(ctx, *p), ctx->gmem_max_rows,
+            small_rows(ctx, *p));
   return GBDTMO_OK;
 }

@@ -12,7 +12,7 @@ namespace gbdtmo {
 // Apply the merged records: decisions for the level's nodes, child nodes, next-level plan.
 __global__ void __launch_bounds__(kPlanThreads)
 k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ xchg, int target_chunks,
-                int64_t gmem_max_rows) {
+                int64_t gmem_max_rows, int64_t small_max_rows) {
   const int64_t LN = int64_t(1) << level, first = LN - 1;
   const int V = channels(p);
   const int64_t RW = rec_words(p);
@@ -49,7 +49,10 @@ k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict_
     const int64_t hs = left_small ? hl : hr, hg = left_small ? hr : hl;
     const bool as = left_small ? al : ar, ag = left_small ? ar : al;
     int32_t ms = MODE_NONE, mg = MODE_NONE;
-    if (ag) { ms = MODE_BUILD; mg = MODE_DERIVE; }      // build the smaller, derive the larger
+    if ((int64_t)(nl > nr ? nl : nr) <= small_max_rows) {   // both small: fused build + search, no subtraction
+      ms = as ? MODE_SMALL : MODE_NONE;
+      mg = ag ? MODE_SMALL : MODE_NONE;
+    } else if (ag) { ms = MODE_BUILD; mg = MODE_DERIVE; }      // build the smaller, derive the larger
     else if (as) { ms = MODE_BUILD; }
     s.node_mode[hs] = ms;
     s.node_mode[hg] = mg;
@@ -211,7 +214,7 @@ extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p,
   int32_t* rows_out = (level & 1) ? s.rows0 : s.rows1;
   const int64_t ntiles = part_tiles(*p);
   GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p),
-            ctx->gmem_max_rows);
+            ctx->gmem_max_rows, small_rows(ctx, *p));
   GB_LAUNCH(k_part_count, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, bm);
   GB_LAUNCH(k_part_scan, 1, kPartThreads, 0, ntiles, s);
   GB_LAUNCH(k_part_scatter, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, rows_out, bm);

@@ -113,6 +113,26 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     s.misc[MISC_GNODE_COUNT] = sh_gn;
     s.misc[MISC_GNODE_ROWS] = sh_gr;
   }
+  __syncthreads();
+  // SMALL nodes (fused build + search) -> their own list
+  __shared__ int sh_sn;
+  if (threadIdx.x == 0) sh_sn = 0;
+  __syncthreads();
+  for (int64_t i0 = 0; i0 < LN; i0 += blockDim.x) {
+    const int64_t i = i0 + threadIdx.x;
+    int take = 0;
+    if (i < LN) take = s.node_mode[first + i] == MODE_SMALL && s.node_state[first + i] == GBDTMO_NODE_ACTIVE;
+    int tn;
+    const int on = block_excl_scan_256(take, &tn);
+    if (take) s.snodes[sh_sn + on] = make_int4((int)i, s.node_begin[first + i], s.node_end[first + i], 0);
+    __syncthreads();
+    if (threadIdx.x == 0) sh_sn += tn;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    s.misc[MISC_SNODE_COUNT] = sh_sn;
+    s.misc[MISC_SWORK_COUNTER] = 0;
+  }
 }
 
 }  // namespace gbdtmo

@@ -12,9 +12,6 @@ namespace gbdtmo {
 constexpr int kFsWarps = 8;      // warps per block = features of one node per block
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 
-__device__ __forceinline__ uint64_t pack_key(double gain, int64_t fb) {
-  return ((uint64_t)__double_as_longlong(gain) & ~0xFFFFFFull) | (uint64_t)(0xFFFFFF - fb);
-}
 
 // Exclusive prefix (over lanes) and total of a per-lane int64.
 __device__ __forceinline__ long long warp_excl(long long x, long long* total) {
@@ -105,7 +102,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
              uint64_t* __restrict__ keys, int write_derived) {
   const int slot = blockIdx.y;
   const int64_t h = (int64_t(1) << level) - 1 + slot;
-  if (s.node_state[h] != GBDTMO_NODE_ACTIVE) return;
+  if (s.node_state[h] != GBDTMO_NODE_ACTIVE || s.node_mode[h] == MODE_SMALL) return;   // SMALL: small.cu
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const bool store = derive && write_derived;
   const bool own = !derive || store;                  // this node's histogram may be written
@@ -192,7 +189,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
         else
           gain = 0.5 * (accL[i] - P);
         if (gain > p.gamma) {
-          const uint64_t key = pack_key(gain, fb0 + b);
+          const uint64_t key = pack_split_key(gain, fb0 + b);
           best = key > best ? key : best;
         }
       }
@@ -228,7 +225,8 @@ __device__ __forceinline__ bool decode_local(const gbdtmo_problem& p, uint64_t k
 }
 
 // One block per slot: left sums at the winning (feature, bin) if the feature is local.
-__global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __restrict__ dflt, State s,
+__global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __restrict__ dflt,
+                               const uint8_t* __restrict__ bins, const int32_t* __restrict__ q, State s,
                                const int64_t* __restrict__ hist,
                                const int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
                                const int32_t* __restrict__ pcnt, const uint64_t* __restrict__ keys,
@@ -250,6 +248,20 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const int db = dflt ? dflt[fl] : -1;            // default bin: recovered from the node totals
   const int64_t* S = s.node_sum + h * (V + 1);
+  if (s.node_mode[h] == MODE_SMALL) {             // not materialised: left sums straight from the rows
+    const int32_t* rl = (level & 1) ? s.rows1 : s.rows0;
+    const int nb0 = s.node_begin[h], nb1 = s.node_end[h];
+    for (int c = warp; c <= V; c += nw) {
+      long long le = 0;
+      for (int pos = nb0 + lane; pos < nb1; pos += 32) {
+        const int r = level > 0 ? rl[pos] : pos;
+        if (bins[(int64_t)r * p.ld_bins + fl] <= b) le += (c < V) ? (long long)q[(int64_t)r * V + c] : 1;
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) le += __shfl_xor_sync(0xffffffffu, le, o);
+      if (lane == 0) rec[c] = le;
+    }
+  } else
   for (int c = warp; c <= V; c += nw) {           // c == V: the counts
     long long le = 0, all = 0;
     for (int bb = lane; bb < B; bb += 32) {
@@ -354,7 +366,8 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
 }
 
 extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
-                                             const uint8_t* bins, const int32_t* dflt, const float* scales, void* state,
+                                             const uint8_t* bins, const int32_t* dflt, const int32_t* q,
+                                             const float* scales, void* state,
                                              const int64_t* hist, const int32_t* cnt,
                                              const int64_t* parent_hist, const int32_t* parent_cnt,
                                              const uint64_t* keys, int64_t* xchg) {
@@ -367,7 +380,7 @@ extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem*
   GB_CHECK_ARG(level == 0 || (parent_hist && parent_cnt), "parent histogram required for level > 0");
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
-  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, s, hist, cnt, level > 0 ? parent_hist : hist,
+  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, bins, q, s, hist, cnt, level > 0 ? parent_hist : hist,
             level > 0 ? parent_cnt : cnt, keys, scales, xchg);
   // zero the record words of the unused slots of this buffer (levels < D-1) so SUM-merging is clean
   const int64_t used = LN * rec_words(*p), cap = bitmap_offset(*p);

@@ -63,7 +63,7 @@ def test_c5_full_size_sampled(orc, pkg):
     del X
     torch.cuda.empty_cache()
     Y = gen.targets_host(w)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(dev), _params(pkg, w, 1))
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(dev), _params(pkg, w, 1), gmem_max_rows=0, small_max_rows=0)
     # --- sampled columns on the host (bit-identical generator) -> oracle binning
     sample = np.array([0, 1, 777, 2048, 4095], np.int64)
     Xs = np.stack([gen.matrix_host(w.seed, gen.STREAM_X, w.x_kind, 0, w.n, int(c), 1, w.m)[:, 0] for c in sample], 1)
@@ -74,7 +74,7 @@ def test_c5_full_size_sampled(orc, pkg):
     for j, c in enumerate(sample):
         np.testing.assert_array_equal(gb[:, int(c)].cpu().numpy(), bins[j])
     # --- level 0 through the ABI, then the root histogram of the sampled features
-    ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+    b._apply_options()
     ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
     b._level(0)
     torch.cuda.synchronize()

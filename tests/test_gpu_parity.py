@@ -127,8 +127,9 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
     rows = node_rows(bins, ref["state"][0], ref["feat"][0], ref["bin"][0], w.n)
     g, h = orc.grad(w.loss, Y.astype(np.float64), np.zeros(Y.shape))
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1), sparse_default=True)
-    ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1), sparse_default=True,
+                    gmem_max_rows=0, small_max_rows=0)
+    b._apply_options()
     ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
     sc = None
     V, B, m, d = b.p.V, w.B, w.m, w.d
@@ -166,17 +167,21 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------- whole trees
 
-@pytest.mark.parametrize("case,sparse,gmem", [("C1", False, 0), ("C2s", False, 0), ("C2s", True, 0), ("C3s", False, 0),
-                                              ("C4s", False, 0), ("C5s", False, 0), ("S300s", False, 0),
-                                              ("C3s", False, 1 << 30), ("C2s", True, 3000), ("C5s", False, 5000)])
-def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem):
+@pytest.mark.parametrize("case,sparse,gmem,small", [
+    ("C1", False, 0, 0), ("C2s", False, 0, 0), ("C2s", True, 0, 0), ("C3s", False, 0, 0), ("C4s", False, 0, 0),
+    ("C5s", False, 0, 0), ("S300s", False, 0, 0),
+    ("C3s", False, 1 << 30, 0), ("C2s", True, 3000, 0), ("C5s", False, 5000, 0),            # global-atomic variant
+    ("C1", False, 0, 2000), ("C2s", False, 0, 4000), ("C2s", True, 256, 2500),               # fused small nodes
+    ("C3s", False, 0, 9000), ("C5s", False, 0, 6000)])
+def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, small):
     w = CASES[case]
     X, Y = _inputs(w)
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
     ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
                     lr=w.lr, min_node=w.min_node)
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse, gmem_max_rows=gmem)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse, gmem_max_rows=gmem,
+                    small_max_rows=small)
     assert (b.dflt is not None) == (sparse and w.index == 2)     # only the MNIST-shaped data has dominant bins
     b.fit()
     torch.cuda.synchronize()
@@ -226,17 +231,18 @@ def test_two_shards_equal_one(orc, pkg, ctx):
     X, Y = _inputs(w)
     Yd = torch.from_numpy(Y).to(DEV)
     P = _params(pkg, w, T=2)
-    full = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), Yd.clone(), P)
+    full = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), Yd.clone(), P,
+                       gmem_max_rows=0, small_max_rows=0)
     full.fit()
     half = w.m // 2 + 3
     shards = []
     for f0, f1 in ((0, half), (half, w.m)):
         ds = pkg.bin_features(ctx, torch.from_numpy(np.ascontiguousarray(X[:, f0:f1])).to(DEV), w.B,
                               f_begin=f0, m_global=w.m)
-        shards.append(pkg.Booster(ctx, ds, Yd.clone(), P))
+        shards.append(pkg.Booster(ctx, ds, Yd.clone(), P, gmem_max_rows=0, small_max_rows=0))
     for t in range(P.T):
         for s in shards:
-            ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
+            s._apply_options()
             ctx.gbdtmo_grad(s.p, s.y, s.pred, s.q, s.scales, s.state)
         for lvl in range(P.D):
             cur, par = lvl % 2, (lvl - 1) % 2
@@ -251,7 +257,7 @@ def test_two_shards_equal_one(orc, pkg, ctx):
                 s.keys.copy_(kmax)
                 ph = s.hist[par] if lvl else None
                 pc = s.cnt[par] if lvl else None
-                ctx.gbdtmo_split_record(s.p, lvl, s.ds.bins, s.dflt, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
+                ctx.gbdtmo_split_record(s.p, lvl, s.ds.bins, s.dflt, s.q, s.scales, s.state, s.hist[cur], s.cnt[cur], ph, pc,
                                         s.keys, s.xchg)
             xs = shards[0].xchg + shards[1].xchg
             for s in shards:

@@ -21,12 +21,13 @@ import paper_conf_icpp_liupw25_b200 as pkg  # noqa: E402
 from gen import gen  # noqa: E402
 
 CANDIDATES = [0, 256, 512, 1024, 2048, 4096, 8192, 16384]
+SMALL_CANDIDATES = [0, 1024, 2048, 4096, 8192, 16384, 32768]
 
 
-def time_trees(ctx, ds, Y, w, thr, warm=2, timed=3):
+def time_trees(ctx, ds, Y, w, thr, small=0, warm=2, timed=3):
     P = pkg.Params(loss=w.loss, T=warm + timed, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
                    min_node=w.min_node)
-    b = pkg.Booster(ctx, ds, Y, P, keep_model=False, gmem_max_rows=thr)
+    b = pkg.Booster(ctx, ds, Y, P, keep_model=False, gmem_max_rows=thr, small_max_rows=small)
     for _ in range(warm):
         b.step()
     torch.cuda.synchronize()
@@ -40,8 +41,8 @@ def time_trees(ctx, ds, Y, w, thr, warm=2, timed=3):
 
 
 def main():
-    shapes = [gen.WORKLOADS["C2"], gen.WORKLOADS["C3"], gen.sweep(5), gen.sweep(100),
-              gen.WORKLOADS["C5"].scaled(n=500_000, m=1024)]
+    shapes = [gen.WORKLOADS["C2"], gen.WORKLOADS["C3"], gen.sweep(5), gen.sweep(10), gen.sweep(50),
+              gen.WORKLOADS["C5"].scaled(n=500_000, m=1024), gen.WORKLOADS["C1"]]
     ctx = pkg.Context(0)
     entries = []
     for w in shapes:
@@ -52,8 +53,12 @@ def main():
         V = w.d * (2 if w.loss == gen.LOSS_SOFTMAX else 1)
         res = {c: time_trees(ctx, ds, Y, w, c) for c in CANDIDATES}
         best = min(res, key=res.get)
+        rs = {c: time_trees(ctx, ds, Y, w, best, c) for c in SMALL_CANDIDATES}
+        best_s = min(rs, key=rs.get)
         entries.append({"workload": w.name, "V": V, "m": w.m, "n": w.n, "gmem_max_rows": best,
-                        "ms_per_tree": {str(k): round(v, 4) for k, v in res.items()}})
+                        "small_max_rows": best_s,
+                        "ms_per_tree": {str(k): round(v, 4) for k, v in res.items()},
+                        "ms_per_tree_small": {str(k): round(v, 4) for k, v in rs.items()}})
         print(json.dumps(entries[-1]), flush=True)
         del ds, Y
         torch.cuda.empty_cache()

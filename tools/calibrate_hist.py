@@ -53,8 +53,12 @@ def main():
         V = w.d * (2 if w.loss == gen.LOSS_SOFTMAX else 1)
         res = {c: time_trees(ctx, ds, Y, w, c) for c in CANDIDATES}
         best = min(res, key=res.get)
+        if res[best] > 0.98 * res[0]:          # noise guard: keep the default unless >= 2% faster
+            best = 0
         rs = {c: time_trees(ctx, ds, Y, w, best, c) for c in SMALL_CANDIDATES}
         best_s = min(rs, key=rs.get)
+        if rs[best_s] > 0.98 * rs[0]:
+            best_s = 0
         entries.append({"workload": w.name, "V": V, "m": w.m, "n": w.n, "gmem_max_rows": best,
                         "small_max_rows": best_s,
                         "ms_per_tree": {str(k): round(v, 4) for k, v in res.items()},

@@ -25,7 +25,9 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-METRIC = "hist rows*outputs/s (sec/tree alongside)"
+# BASELINE.json's metric; `value` is its throughput half (hist rows x outputs per second, whole
+# job), `sec_per_tree` its time half, `roofline.hbm_view` its "% HBM roofline" part.
+METRIC = "sec/tree & hist rows\u00b7outputs/s at 1/2/4/8 B200; % HBM roofline"
 UNIT = "rows*outputs/s"
 
 
@@ -317,7 +319,8 @@ def main():
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps, "warmup": a.warmup,
         "ms_per_step": ms_per_tree, "sec_per_tree": ms_per_tree * 1e-3, "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": None, "dtype": "int64 fixed-point hist / fp64 gains",
+        "scaling": "strong", "vs_baseline": None, "dtype": "int64",
+        "dtype_detail": "31-bit fixed-point g/h, exact int64 histograms, fp64 gains and predictions",
         "data": "synthetic (seeded counter-based generator, gen/); inputs in HBM, 8.2 GB bins >> 126 MB L2 (no flush needed)",
         "config": {"workload": w.name, "n": w.n, "m": w.m, "d": w.d, "B": w.B, "D": w.D,
                    "loss": "mse" if w.loss == 0 else "softmax", "parallelism": f"feature-partition x{world}",

@@ -34,13 +34,14 @@ class Params:
     min_node: int = 20
 
 
-# Measured histogram-variant table (tools/calibrate_hist.py -> profiles/hist_variant_table.json):
-# largest node size (rows) for which the global-atomic variant beat the shared-memory variant,
-# per channel count V.  Empty until calibrated: shared memory everywhere.
+# Measured variant table (tools/calibrate_hist.py -> hist_variant_table.json), per workload shape:
+# gmem_max_rows = largest node (rows) built with the global-atomic histogram variant,
+# small_max_rows = largest pair of siblings searched by sort-and-segment (small.cu) instead of
+# histograms.  0 = off; missing table: shared-memory histograms everywhere.
 _VARIANT_TABLE = None
 
 
-def variant_threshold(V: int, m: int, key: str = "gmem_max_rows") -> int:
+def variant_threshold(V: int, m: int, key: str = "gmem_max_rows", n: Optional[int] = None) -> int:
     global _VARIANT_TABLE
     if _VARIANT_TABLE is None:
         import json
@@ -53,7 +54,11 @@ def variant_threshold(V: int, m: int, key: str = "gmem_max_rows") -> int:
     entries = _VARIANT_TABLE.get("entries", [])
     if not entries:
         return 0
-    e = min(entries, key=lambda e: abs(e["V"] - V))      # nearest measured channel count
+    # nearest measured shape: channel count first, then features and rows (log distance)
+    def dist(e):
+        dn = abs(math.log2(max(n, 1) / max(e.get("n", 1), 1))) if n else 0.0
+        return (abs(math.log2(max(V, 1) / max(e["V"], 1))), abs(math.log2(max(m, 1) / max(e.get("m", 1), 1))) + dn)
+    e = min(entries, key=dist)
     return int(e.get(key, 0))
 
 
@@ -110,8 +115,8 @@ class Booster:
         # histogram variant selection: nodes with <= gmem_max_rows
         # rows use the global-atomic variant; None = the measured table for this channel count
         V = y.shape[1] * (2 if params.loss == LOSS_SOFTMAX else 1)
-        self.gmem_max_rows = variant_threshold(V, ds.m) if gmem_max_rows is None else int(gmem_max_rows)
-        self.small_max_rows = variant_threshold(V, ds.m, "small_max_rows") if small_max_rows is None \
+        self.gmem_max_rows = variant_threshold(V, ds.m, n=ds.n) if gmem_max_rows is None else int(gmem_max_rows)
+        self.small_max_rows = variant_threshold(V, ds.m, "small_max_rows", n=ds.n) if small_max_rows is None \
             else int(small_max_rows)
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.

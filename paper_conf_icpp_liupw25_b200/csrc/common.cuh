@@ -215,10 +215,14 @@ inline const char* check_problem(const gbdtmo_problem* p) {
 
 // Histogram work items wanted per level -> chunks per build level (grad.cu).
 int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p);
-// Whether the fused small-node path fits this problem (small.cu); the effective threshold.
+// Whether the sort-and-segment small-node search fits this problem (small.cu), the largest node
+// its shared-memory staging holds, and the effective threshold min(option, cap).
 bool small_supported(const gbdtmo_problem& p);
+int64_t small_rows_cap(const gbdtmo_problem& p);
 inline int64_t small_rows(const Ctx* ctx, const gbdtmo_problem& p) {
-  return (ctx->small_max_rows > 0 && small_supported(p)) ? ctx->small_max_rows : 0;
+  if (ctx->small_max_rows <= 0 || !small_supported(p)) return 0;
+  const int64_t cap = small_rows_cap(p);
+  return ctx->small_max_rows < cap ? ctx->small_max_rows : cap;
 }
 
 // Launch helpers: count kernels and check errors.

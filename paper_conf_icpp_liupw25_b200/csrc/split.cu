@@ -249,18 +249,32 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   const int db = dflt ? dflt[fl] : -1;            // default bin: recovered from the node totals
   const int64_t* S = s.node_sum + h * (V + 1);
   if (s.node_mode[h] == MODE_SMALL) {             // not materialised: left sums straight from the rows
+    // one pass: warps take 32 rows at a time, lanes = channels sum the rows that go left
+    __shared__ long long acc[2 * 32 + 1];
+    for (int c = threadIdx.x; c <= V; c += blockDim.x) acc[c] = 0;
+    __syncthreads();
     const int32_t* rl = (level & 1) ? s.rows1 : s.rows0;
     const int nb0 = s.node_begin[h], nb1 = s.node_end[h];
-    for (int c = warp; c <= V; c += nw) {
-      long long le = 0;
-      for (int pos = nb0 + lane; pos < nb1; pos += 32) {
-        const int r = level > 0 ? rl[pos] : pos;
-        if (bins[(int64_t)r * p.ld_bins + fl] <= b) le += (c < V) ? (long long)q[(int64_t)r * V + c] : 1;
+    long long a0 = 0, a1 = 0, nleft = 0;
+    for (int pos0 = nb0 + warp * 32; pos0 < nb1; pos0 += nw * 32) {
+      const int pos = pos0 + lane;
+      const int r = pos < nb1 ? (level > 0 ? rl[pos] : pos) : -1;
+      const bool left = r >= 0 && bins[(int64_t)r * p.ld_bins + fl] <= b;
+      unsigned msk = __ballot_sync(0xffffffffu, left);
+      nleft += __popc(msk);
+      while (msk) {
+        const int src = __ffs(msk) - 1;
+        msk &= msk - 1;
+        const int64_t rr = (int64_t)__shfl_sync(0xffffffffu, r, src) * V;
+        if (lane < V) a0 += q[rr + lane];
+        if (lane + 32 < V) a1 += q[rr + lane + 32];
       }
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) le += __shfl_xor_sync(0xffffffffu, le, o);
-      if (lane == 0) rec[c] = le;
     }
+    if (lane < V) atomicAdd((unsigned long long*)&acc[lane], (unsigned long long)a0);
+    if (lane + 32 < V) atomicAdd((unsigned long long*)&acc[lane + 32], (unsigned long long)a1);
+    if (lane == 0) atomicAdd((unsigned long long*)&acc[V], (unsigned long long)nleft);
+    __syncthreads();
+    for (int c = threadIdx.x; c <= V; c += blockDim.x) rec[c] = acc[c];
   } else
   for (int c = warp; c <= V; c += nw) {           // c == V: the counts
     long long le = 0, all = 0;

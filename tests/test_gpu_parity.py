@@ -171,7 +171,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
     ("C1", False, 0, 0), ("C2s", False, 0, 0), ("C2s", True, 0, 0), ("C3s", False, 0, 0), ("C4s", False, 0, 0),
     ("C5s", False, 0, 0), ("S300s", False, 0, 0),
     ("C3s", False, 1 << 30, 0), ("C2s", True, 3000, 0), ("C5s", False, 5000, 0),            # global-atomic variant
-    ("C1", False, 0, 2000), ("C2s", False, 0, 4000), ("C2s", True, 256, 2500),               # fused small nodes
+    ("C1", False, 0, 2000), ("C2s", False, 0, 4000), ("C2s", True, 256, 2500),               # sort-and-segment small nodes
     ("C3s", False, 0, 9000), ("C5s", False, 0, 6000)])
 def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, small):
     w = CASES[case]

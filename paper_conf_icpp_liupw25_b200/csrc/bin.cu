@@ -1,17 +1,15 @@
 // bin.cu — (a)1: per-feature quantile binning ("feature-value bin mapping",
 // "cut points" PAPER.md:166, <= 256 bins PAPER.md:237, 255; exact rule = reading R14).
 //
-// Per tile of TC columns: transpose the column tile into order-preserving uint32 keys,
-// sort every column with a stable 4-pass LSD radix sort (8-bit digits, per-(column, digit,
-// tile) offsets), derive the cuts from the sorted column (distinct values if <= B of them,
-// else the order statistics s[floor(j n / B)]), then bin(x) = #{cuts <= x} by bisection.
+// Per tile of TC columns: transpose the column tile into order-preserving uint32 keys, find
+// per column either its distinct values (if <= B of them) or the order statistics
+// s[floor(j n / B)] by exact most-significant-digit selection (8 counting passes of 4 bits, no
+// key is moved: the column is never sorted), then bin(x) = #{cuts <= x} by bisection.
 #include "common.cuh"
 
 namespace gbdtmo {
 
 constexpr int kBinTC = 64;          // columns per tile
-constexpr int kSortTile = 4096;     // keys per radix block
-constexpr int kSortThreads = 256;
 
 __device__ __forceinline__ uint32_t f2key(float x) {
   uint32_t u = __float_as_uint(x == 0.0f ? 0.0f : x);     // -0.0 == +0.0
@@ -21,9 +19,9 @@ __device__ __forceinline__ float key2f(uint32_t k) {
   return __uint_as_float((k & 0x80000000u) ? (k ^ 0x80000000u) : ~k);
 }
 
-// X[i*ld + c0 + j] -> keys[j*n + i] for j < tc, through a 32x32 shared tile.
+// X[i*ld + c0 + j] -> keys[j*ldk + i] for j < tc, through a 32x32 shared tile.
 __global__ void k_bin_keys(const float* __restrict__ X, int64_t n, int64_t ld_x, int c0, int tc,
-                           uint32_t* __restrict__ keys) {
+                           uint32_t* __restrict__ keys, int64_t ldk) {
   __shared__ uint32_t t[32][33];
   const int64_t i0 = (int64_t)blockIdx.x * 32;
   const int j0 = blockIdx.y * 32;
@@ -36,181 +34,295 @@ __global__ void k_bin_keys(const float* __restrict__ X, int64_t n, int64_t ld_x,
   for (int r = threadIdx.y; r < 32; r += blockDim.y) {
     const int j = j0 + r;
     const int64_t i = i0 + threadIdx.x;
-    if (i < n && j < tc) keys[(int64_t)j * n + i] = t[threadIdx.x][r];
+    if (i < n && j < tc) keys[(int64_t)j * ldk + i] = t[threadIdx.x][r];
   }
 }
 
-// counts[(col*256 + digit)*T + tile] = #keys of the tile with that digit
-__global__ void __launch_bounds__(kSortThreads)
-k_radix_count(const uint32_t* __restrict__ keys, int64_t n, int shift, uint32_t* __restrict__ counts, int64_t T) {
-  __shared__ uint32_t hs[256];
-  const int col = blockIdx.y;
-  const int64_t tile = blockIdx.x;
-  hs[threadIdx.x] = 0;
-  __syncthreads();
-  const uint32_t* kc = keys + (int64_t)col * n;
-  const int64_t beg = tile * kSortTile;
-  for (int j = 0; j < kSortTile / kSortThreads; ++j) {
-    const int64_t pos = beg + j * kSortThreads + threadIdx.x;
-    if (pos < n) atomicAdd(&hs[(kc[pos] >> shift) & 0xFFu], 1u);
-  }
-  __syncthreads();
-  counts[((int64_t)col * 256 + threadIdx.x) * T + tile] = hs[threadIdx.x];
-}
+// ---- exact selection of the order statistics by most-significant-digit refinement.
+//
+// Per column, a sorted list A of at most 256 key prefixes, each with the rank of its first key
+// (base), is refined 4 bits per pass over 8 passes.  A pass counts, for every key whose prefix is
+// in A, the next digit (k_sel_count); k_sel_refine then keeps either every non-empty longer
+// prefix while there are at most B of them ("few" mode: at the end they are the distinct values,
+// rule (i)) or only the prefixes holding one of the ranks 0, floor(j n / B) ("targets" mode: at
+// the end each is the key at that rank, rule (ii)).  Only counters are written: no keys move.
+constexpr int kSelDigits = 16;                 // 4-bit digits
+constexpr int kSelMax = 256;                   // prefixes tracked per column (>= B)
+constexpr int kSelRows = 32768;                // keys per count block
+constexpr int kSelHist = kSelMax * kSelDigits; // counters per column
 
-// In-place exclusive scan of counts[col][0 .. 256*T) (digit-major, tile-minor).
-__global__ void __launch_bounds__(1024) k_radix_scan(uint32_t* __restrict__ counts, int64_t T) {
-  __shared__ uint32_t ws[32];
-  __shared__ uint32_t carry;
+struct SelMeta {
+  int an;      // entries in A
+  int mode;    // 0: few (all non-empty prefixes), 1: targets
+  int pad[2];
+};
+
+__global__ void k_sel_init(int tc, SelMeta* __restrict__ meta, uint32_t* __restrict__ pre, uint32_t* __restrict__ base,
+                           uint32_t* __restrict__ ghist) {
   const int col = blockIdx.x;
-  uint32_t* c = counts + (int64_t)col * 256 * T;
-  const int64_t total = 256 * T;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  if (threadIdx.x == 0) carry = 0;
+  if (threadIdx.x == 0) {
+    meta[col].an = 1; meta[col].mode = 0;
+    pre[col * kSelMax] = 0; base[col * kSelMax] = 0;
+  }
+  for (int e = threadIdx.x; e < kSelHist; e += blockDim.x) ghist[(int64_t)col * kSelHist + e] = 0;
+}
+
+// One counting pass.  pbits = 0: the first pass, counters by the key's top 12 bits (as if A held
+// all 256 8-bit prefixes, 16 digits each).  pbits >= 12: counters of the next 4-bit digit per
+// prefix in A; keys whose prefix is not in A are skipped.  Lookup: a 4096-entry table on the
+// prefix's top 12 bits gives (first entry, entries) of A sharing them, so keys outside A cost one
+// load and the rest a short search.  kout != null: the keys found in A (the only keys later
+// passes can match) are compacted within the block's own slice of kout, their number written to
+// cnt_out[col][block]; cnt_in != null: the block reads only that many keys of its slice.  Each thread
+// takes 8 consecutive keys per step with two 16-byte loads; a warp whose lanes all hit one
+// counter (constant or skewed columns) adds once.
+__global__ void __launch_bounds__(256)
+k_sel_count(const uint32_t* __restrict__ kin, const int32_t* __restrict__ cnt_in, int64_t n, int64_t ldk, int pbits,
+            const SelMeta* __restrict__ meta, const uint32_t* __restrict__ pre, uint32_t* __restrict__ ghist,
+            uint32_t* __restrict__ kout, int32_t* __restrict__ cnt_out) {
+  __shared__ uint32_t sp[kSelMax];
+  __shared__ uint32_t h[kSelHist];
+  __shared__ uint32_t tab[4096];                 // (first << 16) | count, by top-12 bits of the prefix
+  __shared__ int sh_out;
+  const int col = blockIdx.y;
+  const int64_t slot = (int64_t)col * gridDim.x + blockIdx.x;
+  const int64_t beg = (int64_t)blockIdx.x * kSelRows;
+  const int64_t end = cnt_in ? beg + cnt_in[slot] : (beg + kSelRows < n ? beg + kSelRows : n);
+  if (end <= beg) {
+    if (cnt_out && threadIdx.x == 0) cnt_out[slot] = 0;
+    return;
+  }
+  if (threadIdx.x == 0) sh_out = 0;
+  const int an = pbits ? meta[col].an : kSelMax;
+  const int dshift = 28 - pbits;
+  for (int e = threadIdx.x; e < an * kSelDigits; e += blockDim.x) h[e] = 0;
+  if (pbits) {
+    for (int i = threadIdx.x; i < an; i += blockDim.x) sp[i] = pre[col * kSelMax + i];
+    for (int e = threadIdx.x; e < 4096; e += blockDim.x) tab[e] = 0;
+    __syncthreads();
+    for (int i = threadIdx.x; i < an; i += blockDim.x) {     // A is sorted: runs of equal top bits
+      const uint32_t t = sp[i] >> (pbits - 12);
+      if (i == 0 || (sp[i - 1] >> (pbits - 12)) != t) {
+        int k = i + 1;
+        while (k < an && (sp[k] >> (pbits - 12)) == t) ++k;
+        tab[t] = ((uint32_t)i << 16) | (uint32_t)(k - i);
+      }
+    }
+  }
   __syncthreads();
-  for (int64_t b0 = 0; b0 < total; b0 += 1024) {
-    const int64_t i = b0 + threadIdx.x;
-    const uint32_t v = i < total ? c[i] : 0u;
+  const uint32_t* kc = kin + (int64_t)col * ldk;
+  uint32_t* ko = kout ? kout + (int64_t)col * ldk : nullptr;
+  const int lane = threadIdx.x & 31;
+  for (int64_t i0 = beg + 8 * threadIdx.x; i0 - 8 * threadIdx.x < end; i0 += 8 * blockDim.x) {
+    uint32_t k8[8];
+    if (i0 + 8 <= end) {
+      const uint4 a = __ldg(reinterpret_cast<const uint4*>(kc + i0));
+      const uint4 b = __ldg(reinterpret_cast<const uint4*>(kc + i0 + 4));
+      k8[0] = a.x; k8[1] = a.y; k8[2] = a.z; k8[3] = a.w; k8[4] = b.x; k8[5] = b.y; k8[6] = b.z; k8[7] = b.w;
+    } else {
+#pragma unroll
+      for (int u = 0; u < 8; ++u) k8[u] = (i0 + u < end) ? kc[i0 + u] : 0u;
+    }
+    int ev[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      int e = -1;
+      if (i0 + u < end) {
+        const uint32_t key = k8[u];
+        if (!pbits) {
+          e = (int)(key >> 20);
+        } else {
+          const uint32_t kp = key >> (32 - pbits);
+          const uint32_t te = tab[kp >> (pbits - 12)];
+          int lo = (int)(te >> 16), cnt = (int)(te & 0xFFFFu);
+          while (cnt > 1) {                                   // last entry <= kp within the run
+            const int half = cnt >> 1;
+            if (sp[lo + half] <= kp) lo += half;
+            cnt -= half;
+          }
+          if (cnt && sp[lo] == kp) e = lo * kSelDigits + (int)((key >> dshift) & 15u);
+        }
+      }
+      ev[u] = e;
+      // lanes sharing lane 0's counter (a dominant value) add once; the others add their own
+      const int e0 = __shfl_sync(0xffffffffu, e, 0);
+      const unsigned same = __ballot_sync(0xffffffffu, e == e0);
+      if (e == e0) {
+        if (lane == 0 && e0 >= 0) atomicAdd(&h[e0], (uint32_t)__popc(same));
+      } else if (e >= 0) {
+        atomicAdd(&h[e], 1u);
+      }
+    }
+    if (ko) {                                                 // compact the matched keys: one warp scan per 8 keys
+      int mine = 0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) mine += ev[u] >= 0;
+      int x = mine;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) { const int y = __shfl_up_sync(0xffffffffu, x, o); if (lane >= o) x += y; }
+      int wbase = 0;
+      if (lane == 31 && x) wbase = atomicAdd(&sh_out, x);
+      wbase = __shfl_sync(0xffffffffu, wbase, 31) + x - mine;
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (ev[u] >= 0) ko[beg + wbase++] = k8[u];
+    }
+  }
+  __syncthreads();
+  if (cnt_out && threadIdx.x == 0) cnt_out[slot] = sh_out;
+  uint32_t* gh = ghist + (int64_t)col * kSelHist;
+  for (int e = threadIdx.x; e < an * kSelDigits; e += blockDim.x)
+    if (h[e]) atomicAdd(&gh[e], h[e]);
+}
+
+__device__ __forceinline__ uint32_t sel_rank(int j, int64_t n, int B) { return (uint32_t)(((int64_t)j * n) / B); }
+
+// one block of kSelMax threads per column: the next prefix list (and re-zeroed counters)
+__global__ void __launch_bounds__(kSelMax)
+k_sel_refine(int64_t n, int B, int first, SelMeta* __restrict__ meta, uint32_t* __restrict__ pre,
+             uint32_t* __restrict__ base, uint32_t* __restrict__ ghist) {
+  __shared__ uint32_t ws[kSelMax / 32];
+  __shared__ int sh_total;
+  const int col = blockIdx.x, t = threadIdx.x;
+  const int lane = t & 31, w = t >> 5;
+  const int an = first ? kSelMax : meta[col].an, mode = meta[col].mode;
+  uint32_t c[kSelDigits];
+  uint32_t p0 = 0, b0 = 0, tot = 0;
+  uint32_t* gh = ghist + (int64_t)col * kSelHist;
+  if (t < an) {
+    p0 = first ? (uint32_t)t : pre[col * kSelMax + t];        // first pass: A = all 8-bit prefixes
+    b0 = first ? 0u : base[col * kSelMax + t];
+#pragma unroll
+    for (int d = 0; d < kSelDigits; ++d) { c[d] = gh[t * kSelDigits + d]; gh[t * kSelDigits + d] = 0; tot += c[d]; }
+  } else {
+#pragma unroll
+    for (int d = 0; d < kSelDigits; ++d) c[d] = 0;
+  }
+  // block exclusive scan helper (kSelMax threads)
+  auto scan = [&](uint32_t v) -> uint32_t {
     uint32_t x = v;
-    for (int o = 1; o < 32; o <<= 1) { uint32_t y = __shfl_up_sync(0xffffffffu, x, o); if (lane >= o) x += y; }
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) { const uint32_t y = __shfl_up_sync(0xffffffffu, x, o); if (lane >= o) x += y; }
     if (lane == 31) ws[w] = x;
     __syncthreads();
-    if (w == 0) {
-      uint32_t s = ws[lane];
-      for (int o = 1; o < 32; o <<= 1) { uint32_t y = __shfl_up_sync(0xffffffffu, s, o); if (lane >= o) s += y; }
-      ws[lane] = s;
+    if (t == 0) {
+      uint32_t acc = 0;
+      for (int k = 0; k < kSelMax / 32; ++k) { const uint32_t q = ws[k]; ws[k] = acc; acc += q; }
+      sh_total = (int)acc;
     }
     __syncthreads();
-    const uint32_t base = (w ? ws[w - 1] : 0u) + carry;
-    if (i < total) c[i] = base + x - v;
+    const uint32_t r = ws[w] + x - v;
     __syncthreads();
-    if (threadIdx.x == 0) carry += ws[31];
-    __syncthreads();
-  }
-}
-
-// Stable scatter: the tile is consumed in rounds of 256 consecutive keys; ranks inside a round
-// come from warp match + per-(warp, digit) counts, so equal digits keep their input order.
-__global__ void __launch_bounds__(kSortThreads)
-k_radix_scatter(const uint32_t* __restrict__ kin, uint32_t* __restrict__ kout, int64_t n, int shift,
-                const uint32_t* __restrict__ counts, int64_t T) {
-  constexpr int NW = kSortThreads / 32;
-  __shared__ uint32_t base[256];
-  __shared__ uint32_t run[256];
-  __shared__ uint32_t wcnt[NW][256];
-  __shared__ uint32_t woff[NW][256];
-  const int col = blockIdx.y;
-  const int64_t tile = blockIdx.x;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  base[threadIdx.x] = counts[((int64_t)col * 256 + threadIdx.x) * T + tile];
-  run[threadIdx.x] = 0;
-  for (int x = 0; x < NW; ++x) wcnt[x][threadIdx.x] = 0;
-  __syncthreads();
-  const uint32_t* kc = kin + (int64_t)col * n;
-  uint32_t* ko = kout + (int64_t)col * n;
-  const uint32_t lt = (1u << lane) - 1u;
-  for (int rd = 0; rd < kSortTile / kSortThreads; ++rd) {
-    const int64_t pos = tile * kSortTile + (int64_t)rd * kSortThreads + threadIdx.x;
-    const bool on = pos < n;
-    const uint32_t key = on ? kc[pos] : 0u;
-    const int dig = on ? (int)((key >> shift) & 0xFFu) : 256;
-    const uint32_t peers = __match_any_sync(0xffffffffu, dig);
-    const int rank = __popc(peers & lt);
-    if (on && rank == 0) wcnt[w][dig] = __popc(peers);
-    __syncthreads();
-    {
-      const int t = threadIdx.x;
-      uint32_t acc = run[t];
-      for (int x = 0; x < NW; ++x) { const uint32_t cx = wcnt[x][t]; woff[x][t] = acc; acc += cx; wcnt[x][t] = 0; }
-      run[t] = acc;
+    return r;
+  };
+  if (first) b0 = scan(tot);
+  uint32_t nzmask = 0;
+#pragma unroll
+  for (int d = 0; d < kSelDigits; ++d) nzmask |= (c[d] ? 1u : 0u) << d;
+  uint32_t off = scan((uint32_t)__popc(nzmask));
+  const int N = sh_total;
+  uint32_t keep = nzmask;
+  int new_mode = mode;
+  if (mode == 1 || N > B) {
+    new_mode = 1;                                  // keep the prefixes holding a target rank
+    keep = 0;
+    if (t < an && tot) {
+      const uint32_t lo = b0, hi = b0 + tot;       // ranks [lo, hi)
+      int j = (int)(((int64_t)lo * B) / n);
+      while (j > 0 && sel_rank(j, n, B) >= lo) --j;
+      while (j < B && sel_rank(j, n, B) < lo) ++j;
+      for (; j < B && sel_rank(j, n, B) < hi; ++j) {
+        const uint32_t r = sel_rank(j, n, B) - lo;
+        uint32_t acc = 0;
+        int d = 0;
+        while (acc + c[d] <= r) { acc += c[d]; ++d; }
+        keep |= 1u << d;
+      }
     }
-    __syncthreads();
-    if (on) ko[base[dig] + woff[w][dig] + rank] = key;
-    __syncthreads();
+    off = scan((uint32_t)__popc(keep));
   }
+  const int total = sh_total;
+  if (t < an) {
+    uint32_t acc = b0, k = off;
+#pragma unroll
+    for (int d = 0; d < kSelDigits; ++d) {
+      if ((keep >> d) & 1u) {
+        pre[col * kSelMax + k] = (p0 << 4) | (uint32_t)d;
+        base[col * kSelMax + k] = acc;
+        ++k;
+      }
+      acc += c[d];
+    }
+  }
+  if (t == 0) { meta[col].an = total; meta[col].mode = new_mode; }
 }
 
-// One block per column of the sorted tile: cuts and nbins (reading R14).
-__global__ void __launch_bounds__(1024)
-k_bin_cuts(const uint32_t* __restrict__ keys, int64_t n, int B, float* __restrict__ cuts, int32_t* __restrict__ nbins) {
-  __shared__ uint32_t ws[32];
-  __shared__ uint32_t sh_total, carry;
+// cuts and nbins from the final (full-key) list (reading R14)
+__global__ void k_sel_cuts(int64_t n, int B, const SelMeta* __restrict__ meta, const uint32_t* __restrict__ pre,
+                           const uint32_t* __restrict__ base, float* __restrict__ cuts, int32_t* __restrict__ nbins) {
   const int col = blockIdx.x;
-  const uint32_t* s = keys + (int64_t)col * n;
   float* cut = cuts + (int64_t)col * (B - 1);
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  // distinct count (capped: we only need to know whether it is <= B)
-  uint32_t local = 0;
-  for (int64_t i = 1 + threadIdx.x; i < n; i += blockDim.x) local += s[i] != s[i - 1];
-  for (int o = 16; o > 0; o >>= 1) local += __shfl_xor_sync(0xffffffffu, local, o);
-  if (threadIdx.x == 0) sh_total = 0;
-  __syncthreads();
-  if (lane == 0) atomicAdd(&sh_total, local);
   for (int j = threadIdx.x; j < B - 1; j += blockDim.x) cut[j] = __int_as_float(0x7f800000);   // +inf
   __syncthreads();
-  const uint64_t distinct = (uint64_t)sh_total + 1;
-  if (distinct <= (uint64_t)B) {
-    // rule (i): every distinct value except the smallest, in order
-    if (threadIdx.x == 0) carry = 0;
-    __syncthreads();
-    for (int64_t b0 = 1; b0 < n; b0 += blockDim.x) {
-      const int64_t i = b0 + threadIdx.x;
-      const uint32_t f = (i < n && s[i] != s[i - 1]) ? 1u : 0u;
-      uint32_t x = f;
-      for (int o = 1; o < 32; o <<= 1) { uint32_t y = __shfl_up_sync(0xffffffffu, x, o); if (lane >= o) x += y; }
-      if (lane == 31) ws[w] = x;
-      __syncthreads();
-      if (w == 0) {
-        uint32_t t = ws[lane];
-        for (int o = 1; o < 32; o <<= 1) { uint32_t y = __shfl_up_sync(0xffffffffu, t, o); if (lane >= o) t += y; }
-        ws[lane] = t;
-      }
-      __syncthreads();
-      const uint32_t off = carry + (w ? ws[w - 1] : 0u) + x - f;
-      if (f) cut[off] = key2f(s[i]);
-      __syncthreads();
-      if (threadIdx.x == 0) carry += ws[31];
-      __syncthreads();
-    }
-    if (threadIdx.x == 0) nbins[col] = (int32_t)distinct;
-  } else if (threadIdx.x == 0) {
-    // rule (ii): order statistics s[floor(j n / B)], deduplicated, those <= s[0] dropped
-    const float s0 = key2f(s[0]);
-    int k = 0;
-    float last = 0.0f;
-    for (int j = 1; j <= B - 1; ++j) {
-      const float v = key2f(s[((int64_t)j * n) / B]);
-      if (v <= s0) continue;
-      if (k > 0 && v == last) continue;
-      cut[k++] = v;
-      last = v;
-    }
-    nbins[col] = k + 1;
+  if (threadIdx.x) return;
+  const int an = meta[col].an;
+  const uint32_t* P = pre + col * kSelMax;
+  const uint32_t* R = base + col * kSelMax;
+  if (meta[col].mode == 0) {                       // rule (i): every distinct value but the smallest
+    for (int k = 1; k < an; ++k) cut[k - 1] = key2f(P[k]);
+    nbins[col] = an;
+    return;
   }
+  // rule (ii): s[floor(j n / B)], j = 1..B-1, deduplicated, those <= s[0] dropped
+  const uint32_t s0 = P[0];
+  int k = 0, e = 0;
+  uint32_t last = 0;
+  for (int j = 1; j <= B - 1; ++j) {
+    const uint32_t r = sel_rank(j, n, B);
+    while (e + 1 < an && R[e + 1] <= r) ++e;      // last entry starting at or before rank r
+    const uint32_t v = P[e];
+    if (v <= s0) continue;
+    if (k > 0 && v == last) continue;
+    cut[k++] = key2f(v);
+    last = v;
+  }
+  nbins[col] = k + 1;
 }
 
-// bins[i*ld + c0 + j] = #{cuts_j <= X[i, c0 + j]}
-__global__ void k_bin_apply(const float* __restrict__ X, int64_t n, int64_t ld_x, int c0, int tc, int B,
-                            const float* __restrict__ cuts, const int32_t* __restrict__ nbins,
-                            uint8_t* __restrict__ bins, int64_t ld_bins) {
+// bins[i*ld + c0 + j] = #{cuts_j <= X[i, c0 + j]}: lanes over the tile's columns, rows strided.
+// 1024-thread blocks (two per SM share the 64-column cut table's 65 KB each) and 4 rows per
+// thread keep enough loads in flight: the kernel is bound by the latency of X.
+constexpr int kApplyThreads = 1024;
+__global__ void __launch_bounds__(kApplyThreads)
+k_bin_apply(const float* __restrict__ X, int64_t n, int64_t ld_x, int c0, int tc, int B,
+            const float* __restrict__ cuts, const int32_t* __restrict__ nbins, uint8_t* __restrict__ bins,
+            int64_t ld_bins) {
   extern __shared__ float sc[];          // [tc][B-1]
-  __shared__ int nb[kBinTC];
+  __shared__ int nc[kBinTC];
   for (int e = threadIdx.x; e < tc * (B - 1); e += blockDim.x) sc[e] = cuts[(int64_t)c0 * (B - 1) + e];
-  for (int j = threadIdx.x; j < tc; j += blockDim.x) nb[j] = nbins[c0 + j];
+  for (int j = threadIdx.x; j < tc; j += blockDim.x) nc[j] = nbins[c0 + j] - 1;
   __syncthreads();
-  const int64_t total = n * tc;
-  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t i = e / tc;
-    const int j = (int)(e - i * tc);
-    const float x = X[i * ld_x + c0 + j];
-    const float* c = sc + j * (B - 1);
-    int lo = 0, hi = nb[j] - 1;
-    while (lo < hi) { const int mid = (lo + hi) >> 1; if (c[mid] <= x) lo = mid + 1; else hi = mid; }
-    bins[i * ld_bins + c0 + j] = (uint8_t)lo;
+  const int j = threadIdx.x % kBinTC, r0 = threadIdx.x / kBinTC;
+  constexpr int RPB = kApplyThreads / kBinTC;   // rows per block iteration
+  if (j >= tc) return;
+  const float* c = sc + j * (B - 1);
+  const int ncut = nc[j];
+  constexpr int U = 4;                   // rows per thread per step (loads issued first)
+  const int64_t step = (int64_t)gridDim.x * RPB;
+  for (int64_t i = (int64_t)blockIdx.x * RPB + r0; i < n; i += U * step) {
+    float x[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) x[u] = (i + u * step < n) ? __ldg(&X[(i + u * step) * ld_x + c0 + j]) : 0.0f;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      int lo = 0;                        // #cuts <= x (ncut <= 255)
+#pragma unroll
+      for (int st = 128; st > 0; st >>= 1)
+        if (lo + st <= ncut && c[lo + st - 1] <= x[u]) lo += st;
+      if (i + u * step < n) bins[(i + u * step) * ld_bins + c0 + j] = (uint8_t)lo;
+    }
   }
 }
-
-inline int64_t sort_tiles(int64_t n) { return (n + kSortTile - 1) / kSortTile; }
 
 // dflt[f] = most frequent bin of feature f (ties: smallest).  One block per 8 features (one
 // aligned 8-byte load per row), per-feature shared counters.
@@ -249,10 +361,12 @@ __global__ void __launch_bounds__(256) k_default_bins(const uint8_t* __restrict_
 
 using namespace gbdtmo;
 
+// workspace: keys, compacted keys [tc][ldk] u32 | meta [tc] | prefixes, bases [tc][kSelMax] u32 | counters [tc][kSelHist] u32
 extern "C" size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B) {
   (void)B;
   const int64_t tc = m < kBinTC ? m : kBinTC;
-  return (size_t)(2 * tc * n * 4 + tc * 256 * sort_tiles(n) * 4 + 1024);
+  return (size_t)(2 * tc * ((n + 3) / 4 * 4) * 4 + tc * (int64_t)sizeof(SelMeta) + 2 * tc * kSelMax * 4 + tc * kSelHist * 4 +
+                  2 * tc * ((n + kSelRows - 1) / kSelRows) * 4 + 1024);
 }
 
 extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t B,
@@ -261,16 +375,23 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
   Ctx* ctx = (Ctx*)c;
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X && bins && cuts && nbins && ws, "null pointer");
+  GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
   GB_CHECK_ARG(n >= 1 && n < (int64_t(1) << 31) && m >= 1, "bad n or m");
   GB_CHECK_ARG(ld_x >= m && ld_bins >= m, "bad leading dimension");
   if (B > 256) { ctx->err = "gbdtmo_bin: B > 256 unsupported (bins are uint8)"; return GBDTMO_EUNSUPPORTED; }
   GB_CHECK_ARG(B >= 2, "B < 2");
   if (ws_bytes < gbdtmo_bin_workspace_bytes(n, m, B)) { ctx->err = "gbdtmo_bin: workspace too small"; return GBDTMO_ENOMEM; }
   const int64_t tcmax = m < kBinTC ? m : kBinTC;
-  const int64_t T = sort_tiles(n);
+  const int64_t ldk = (n + 3) / 4 * 4;                    // 16-byte aligned key columns
   uint32_t* ka = (uint32_t*)ws;
-  uint32_t* kb = ka + tcmax * n;
-  uint32_t* counts = kb + tcmax * n;
+  uint32_t* kb = ka + tcmax * ldk;
+  SelMeta* meta = (SelMeta*)(kb + tcmax * ldk);
+  uint32_t* pre = (uint32_t*)(meta + tcmax);
+  uint32_t* base = pre + tcmax * kSelMax;
+  uint32_t* ghist = base + tcmax * kSelMax;
+  const unsigned row_blocks = (unsigned)((n + kSelRows - 1) / kSelRows);
+  int32_t* cnt_a = (int32_t*)(ghist + tcmax * kSelHist);    // kept keys per (column, block)
+  int32_t* cnt_b = cnt_a + tcmax * row_blocks;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(k_bin_apply, cudaFuncAttributeMaxDynamicSharedMemorySize, kBinTC * 255 * 4);
@@ -278,17 +399,24 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
   }
   for (int c0 = 0; c0 < m; c0 += kBinTC) {
     const int tc = (int)(m - c0 < kBinTC ? m - c0 : kBinTC);
-    GB_LAUNCH(k_bin_keys, dim3((unsigned)((n + 31) / 32), (unsigned)((tc + 31) / 32)), dim3(32, 8), 0, X, n, ld_x, c0, tc, ka);
-    uint32_t* kin = ka;
-    uint32_t* kout = kb;
-    for (int pass = 0; pass < 4; ++pass) {
-      GB_LAUNCH(k_radix_count, dim3((unsigned)T, (unsigned)tc), kSortThreads, 0, kin, n, 8 * pass, counts, T);
-      GB_LAUNCH(k_radix_scan, (unsigned)tc, 1024, 0, counts, T);
-      GB_LAUNCH(k_radix_scatter, dim3((unsigned)T, (unsigned)tc), kSortThreads, 0, kin, kout, n, 8 * pass, counts, T);
-      uint32_t* t = kin; kin = kout; kout = t;
+    GB_LAUNCH(k_bin_keys, dim3((unsigned)((n + 31) / 32), (unsigned)((tc + 31) / 32)), dim3(32, 8), 0, X, n, ld_x, c0, tc, ka, ldk);
+    GB_LAUNCH(k_sel_init, (unsigned)tc, 256, 0, tc, meta, pre, base, ghist);
+    // prefix bits before each pass: 0 (12-bit digit), then 12, 16, 20, 24, 28 (4-bit digits);
+    // from 16 bits on, the matched keys are compacted and only they are read by the next pass
+    const int pb[6] = {0, 12, 16, 20, 24, 28};
+    for (int k = 0; k < 6; ++k) {
+      const bool rd_c = pb[k] >= 20, wr_c = pb[k] >= 16 && pb[k] <= 24;
+      const uint32_t* kin = (pb[k] == 20 || pb[k] == 28) ? kb : ka;
+      uint32_t* kout = wr_c ? (pb[k] == 20 ? ka : kb) : nullptr;
+      const int32_t* cin = rd_c ? ((pb[k] == 24) ? cnt_b : cnt_a) : nullptr;
+      int32_t* cout = wr_c ? ((pb[k] == 20) ? cnt_b : cnt_a) : nullptr;
+      GB_LAUNCH(k_sel_count, dim3(row_blocks, (unsigned)tc), 256, 0, kin, cin, n, ldk, pb[k], meta, pre, ghist, kout,
+                cout);
+      GB_LAUNCH(k_sel_refine, (unsigned)tc, kSelMax, 0, n, B, (int)(pb[k] == 0), meta, pre, base, ghist);
     }
-    GB_LAUNCH(k_bin_cuts, (unsigned)tc, 1024, 0, kin, n, B, cuts + (int64_t)c0 * (B - 1), nbins + c0);
-    GB_LAUNCH(k_bin_apply, ctx->num_sms * 4, 256, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts, nbins, bins, ld_bins);
+    GB_LAUNCH(k_sel_cuts, (unsigned)tc, 256, 0, n, B, meta, pre, base, cuts + (int64_t)c0 * (B - 1), nbins + c0);
+    GB_LAUNCH(k_bin_apply, ctx->num_sms * 2, kApplyThreads, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts, nbins, bins,
+              ld_bins);
   }
   return GBDTMO_OK;
 }

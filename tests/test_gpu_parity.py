@@ -84,6 +84,29 @@ def test_bin_edge_cases(orc, pkg, ctx):
         np.testing.assert_array_equal(gb.T, bins)
 
 
+@pytest.mark.parametrize("n", [1, 2, 3, 7, 257, 8193, 20011])
+def test_bin_selection_edge_cases(orc, pkg, ctx, n):
+    """Exact order statistics by digit selection: ragged n, exactly B / B+1 distinct values,
+    duplicates straddling target ranks, mixed signs, denormals and huge magnitudes."""
+    rng = np.random.default_rng(n)
+    cols = [
+        rng.integers(0, 256, n), rng.integers(0, 257, n),                        # B and B+1 distinct
+        np.repeat(rng.normal(size=(n + 9) // 10), 10)[:n],                        # runs of 10 equal values
+        rng.normal(size=n) * np.float32(1e-40), rng.normal(size=n) * 1e30,        # denormal / huge
+        np.where(rng.random(n) < 0.9, 0.0, rng.normal(size=n)),                   # 90 % zeros
+        -np.abs(rng.standard_cauchy(n)), rng.random(n).astype(np.float32) + 1.0,  # heavy tail; one exponent
+    ] + [rng.normal(size=n) for _ in range(60)]                                   # > 64 columns: two tiles
+    X = np.stack(cols, axis=1).astype(np.float32)
+    for B in (2, 255, 256):
+        ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), B)
+        torch.cuda.synchronize()
+        cuts, nbins, bins = orc.bin_matrix(X, B)
+        np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+        np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+        gb = ds.bins[: n * ds.ld_bins].view(n, ds.ld_bins)[:, : X.shape[1]].cpu().numpy()
+        np.testing.assert_array_equal(gb.T, bins)
+
+
 # ------------------------------------------------------------------------- gradients
 
 @pytest.mark.parametrize("case", ["C1", "C2s"])

@@ -143,6 +143,21 @@ gbdtmo_status gbdtmo_bin(gbdtmo_ctx ctx, const float* X, int64_t n, int32_t m, i
                          uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                          void* ws, size_t ws_bytes);
 
+/* The same binning from the paper's sparse storage (Compressed Sparse Column:
+ * "values", "row_indices", "col_pointers"; entries not stored are 0).  Result identical to
+ * gbdtmo_bin on the dense matrix.  The implicit zeros are never materialised: they join the
+ * selection counts per column and fill the bins before the stored values are scattered.
+ * values       float32 [nnz] (device), column by column; explicit zeros allowed
+ * row_idx      int32 [nnz] (device), row of each value; at most one entry per (row, column)
+ *              (duplicates: undefined result)
+ * col_ptr      int64 [m+1] (device), column j holds entries [col_ptr[j], col_ptr[j+1])
+ * col_ptr_host the same array in host memory (validated; sizes the launches)
+ * bins, cuts, nbins, ws as for gbdtmo_bin (ws of gbdtmo_bin_workspace_bytes(n, m, B) bytes).
+ * EINVAL if col_ptr[0] != 0, it decreases, or a column holds more than n entries. */
+gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx ctx, const float* values, const int32_t* row_idx, const int64_t* col_ptr,
+                             const int64_t* col_ptr_host, int64_t n, int32_t m, int32_t B, uint8_t* bins,
+                             int64_t ld_bins, float* cuts, int32_t* nbins, void* ws, size_t ws_bytes);
+
 /* Sparsity-aware default bins (zeros are implicit in the paper's CSC
  * storage; here every feature's most frequent bin plays that role): dflt[f] = the bin of feature
  * f holding the most of the n rows (ties: smallest bin), or -1 when that bin holds fewer than

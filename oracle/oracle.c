@@ -49,6 +49,34 @@ static int32_t count_cuts_le(const float* cuts, int32_t ncuts, float x) {
  *   (i)  <= B distinct values: cuts = every distinct value except the smallest.
  *   (ii) otherwise: c_j = s[floor(j*n/B)], j = 1..B-1, duplicates dropped, and every c <= s[0] dropped.
  *   nbins = #cuts + 1. */
+/* "For non-zero values, we traverse the matrix column-wise", "For row indices,
+ * we store the row number of each non-zero value", "The column pointer array has an additional
+ * element indicating the end of the last column". */
+void oracle_csc_from_dense(const float* X, int64_t n, int32_t m, int64_t ld_x,
+                           float* values, int32_t* row_idx, int64_t* col_ptr) {
+  int64_t p = 0;
+  for (int32_t j = 0; j < m; ++j) {
+    col_ptr[j] = p;
+    for (int64_t i = 0; i < n; ++i) {
+      const float x = X[i * ld_x + j];
+      if (x != 0.0f) {
+        if (values) values[p] = x;
+        if (row_idx) row_idx[p] = (int32_t)i;
+        ++p;
+      }
+    }
+  }
+  col_ptr[m] = p;
+}
+
+void oracle_dense_from_csc(const float* values, const int32_t* row_idx, const int64_t* col_ptr,
+                           int64_t n, int32_t m, int64_t ld_x, float* X) {
+  for (int64_t i = 0; i < n; ++i)
+    for (int32_t j = 0; j < m; ++j) X[i * ld_x + j] = 0.0f;
+  for (int32_t j = 0; j < m; ++j)
+    for (int64_t p = col_ptr[j]; p < col_ptr[j + 1]; ++p) X[(int64_t)row_idx[p] * ld_x + j] = values[p];
+}
+
 void oracle_bin(const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t B,
                 float* cuts, int32_t* nbins, uint16_t* bins_cm) {
 #pragma omp parallel for schedule(dynamic, 1)

@@ -18,6 +18,8 @@
  *
  * Parity status per function:
  *   oracle_bin            pinned  (closed form on permutations; distinct-value rank)
+ *   oracle_csc_from_dense pinned  (the paper's worked example, tests/golden/)
+ *   oracle_dense_from_csc pinned  (same example; round trip)
  *   oracle_grad           pinned  (finite differences of the loss; softmax invariants)
  *   oracle_build_hist     pinned  (row-sum invariants, exact dyadic parent = L + R, brute force)
  *   oracle_find_split     pinned  (exhaustive raw-threshold enumeration; sklearn CART, MSE λ=0)
@@ -42,6 +44,16 @@ enum { ORACLE_LOSS_MSE = 0, ORACLE_LOSS_SOFTMAX = 1 };
  * +inf padded), nbins[f] = #cuts + 1, bins_cm[f*n + i] = #{cuts of f <= X(i,f)}. */
 void oracle_bin(const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t B,
                 float* cuts, int32_t* nbins, uint16_t* bins_cm);
+
+/* Compressed Sparse Column storage (§3.2): traverse the matrix column-wise;
+ * values = the non-zero entries, row_idx = their rows, col_ptr[j] = index in values where column
+ * j starts, col_ptr[m] = number of non-zeros.  X row-major, element (i, f) at X[i*ld_x + f].
+ * Pass values = row_idx = NULL to obtain col_ptr only (the sizes). */
+void oracle_csc_from_dense(const float* X, int64_t n, int32_t m, int64_t ld_x,
+                           float* values, int32_t* row_idx, int64_t* col_ptr);
+/* The inverse: X (row-major, ld_x) = 0 everywhere, then X(row_idx[p], j) = values[p]. */
+void oracle_dense_from_csc(const float* values, const int32_t* row_idx, const int64_t* col_ptr,
+                           int64_t n, int32_t m, int64_t ld_x, float* X);
 
 /* Per-output first/second derivatives (PAPER.md:164 MSE; R12 softmax-CE; R13 diagonal H). */
 void oracle_grad(int32_t loss, const double* y, const double* pred, int64_t n, int32_t d,

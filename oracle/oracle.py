@@ -46,6 +46,8 @@ def lib():
         P = C.c_void_p
         i32, i64, f64 = C.c_int32, C.c_int64, C.c_double
         _LIB.oracle_bin.argtypes = [P, i64, i32, i64, i32, P, P, P]
+        _LIB.oracle_csc_from_dense.argtypes = [P, i64, i32, i64, P, P, P]
+        _LIB.oracle_dense_from_csc.argtypes = [P, P, P, i64, i32, i64, P]
         _LIB.oracle_grad.argtypes = [i32, P, P, i64, i32, P, P]
         _LIB.oracle_build_hist.argtypes = [P, i64, i32, i32, P, P, i32, P, i64, P, P, P]
         _LIB.oracle_gain.argtypes = [P, P, P, P, i32, f64]
@@ -81,6 +83,27 @@ def bin_matrix(X, B):
     bins = np.empty((m, n), np.uint16)
     lib().oracle_bin(_p(X), n, m, m, B, _p(cuts), _p(nbins), _p(bins))
     return cuts, nbins, bins
+
+
+def csc_from_dense(X):
+    """X float32 [n][m] -> (values f32 [nnz], row_idx i32 [nnz], col_ptr i64 [m+1])."""
+    X = _c(X, np.float32)
+    n, m = X.shape
+    col_ptr = np.empty(m + 1, np.int64)
+    lib().oracle_csc_from_dense(_p(X), n, m, m, None, None, _p(col_ptr))
+    nnz = int(col_ptr[m])
+    values = np.empty(nnz, np.float32)
+    row_idx = np.empty(nnz, np.int32)
+    lib().oracle_csc_from_dense(_p(X), n, m, m, _p(values), _p(row_idx), _p(col_ptr))
+    return values, row_idx, col_ptr
+
+
+def dense_from_csc(values, row_idx, col_ptr, n):
+    values = _c(values, np.float32); row_idx = _c(row_idx, np.int32); col_ptr = _c(col_ptr, np.int64)
+    m = len(col_ptr) - 1
+    X = np.empty((n, m), np.float32)
+    lib().oracle_dense_from_csc(_p(values), _p(row_idx), _p(col_ptr), n, m, m, _p(X))
+    return X
 
 
 def grad(loss, y, pred):

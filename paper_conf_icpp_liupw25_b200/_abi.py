@@ -25,7 +25,7 @@ SYMBOLS = (
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
-    "gbdtmo_set_option", "gbdtmo_search_small",
+    "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS = 1, 2
 
@@ -71,6 +71,7 @@ def lib():
             "gbdtmo_hist_bytes": ([PP, i32, C.POINTER(sz), C.POINTER(sz)], C.c_int),
             "gbdtmo_xchg_count": ([PP, C.POINTER(i64)], C.c_int),
             "gbdtmo_bin": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz], C.c_int),
+            "gbdtmo_bin_csc": ([P, P, P, P, P, i64, i32, i32, P, i64, P, P, P, sz], C.c_int),
             "gbdtmo_grad": ([P, PP, P, P, P, P, P], C.c_int),
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
@@ -166,6 +167,12 @@ class Context:
         return int(v.value)
 
     # the hot-path calls --------------------------------------------------------
+    def gbdtmo_bin_csc(self, values, row_idx, col_ptr, col_ptr_host, n, m, B, bins, ld_bins, cuts, nbins, ws,
+                       ws_bytes):
+        self._check(lib().gbdtmo_bin_csc(self._h, _ptr(values), _ptr(row_idx), _ptr(col_ptr), _ptr(col_ptr_host), n,
+                                         m, B, _ptr(bins), ld_bins, _ptr(cuts), _ptr(nbins), _ptr(ws), ws_bytes),
+                    "gbdtmo_bin_csc")
+
     def gbdtmo_bin(self, X, n, m, ld_x, B, bins, ld_bins, cuts, nbins, ws, ws_bytes):
         self._check(lib().gbdtmo_bin(self._h, _ptr(X), n, m, ld_x, B, _ptr(bins), ld_bins, _ptr(cuts),
                                      _ptr(nbins), _ptr(ws), ws_bytes), "gbdtmo_bin")

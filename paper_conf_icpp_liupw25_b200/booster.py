@@ -104,6 +104,32 @@ def bin_features(ctx: Context, X: torch.Tensor, B: int, f_begin: int = 0, m_glob
     return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt)
 
 
+def bin_features_csc(ctx: Context, values: torch.Tensor, row_idx: torch.Tensor, col_ptr: torch.Tensor, n: int,
+                     B: int, f_begin: int = 0, m_global: Optional[int] = None) -> Dataset:
+    """gbdtmo_bin_csc on the paper's sparse storage: values float32 [nnz],
+    row_idx int32 [nnz] (device), col_ptr int64 [m+1] (host or device).  Same Dataset as
+    bin_features on the dense matrix."""
+    cp_host = col_ptr.detach().to("cpu", torch.int64).contiguous()
+    dev = values.device
+    assert values.is_cuda and values.dtype == torch.float32 and row_idx.dtype == torch.int32
+    cp_dev = cp_host.to(dev)
+    m = cp_host.numel() - 1
+    ld = _align(m, 16)
+    bins = torch.empty(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
+    cuts = torch.empty((m, B - 1), dtype=torch.float32, device=dev)
+    nbins = torch.empty(m, dtype=torch.int32, device=dev)
+    wsb = ctx.gbdtmo_bin_workspace_bytes(n, m, B)
+    ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
+    ctx.gbdtmo_bin_csc(values if values.numel() else None, row_idx if row_idx.numel() else None, cp_dev, cp_host,
+                       n, m, B, bins, ld, cuts, nbins, ws, wsb)
+    dflt = torch.empty(m, dtype=torch.int32, device=dev)
+    ctx.gbdtmo_default_bins(bins, n, m, ld, B, max(1, n // 16), dflt)
+    if not bool((dflt >= 0).any()):
+        dflt = None
+    return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt)
+
+
 class Booster:
     """One GBDT-MO model being trained on one GPU (one feature shard when `group` is given)."""
 

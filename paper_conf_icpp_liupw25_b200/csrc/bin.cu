@@ -357,16 +357,148 @@ __global__ void __launch_bounds__(256) k_default_bins(const uint8_t* __restrict_
   }
 }
 
+// ---- CSC input (values, row indices, column pointers; absent entries are 0)
+
+// keys of the tile's stored values, column by column (ka[j*ldk + i], i < nnz_j); per column the
+// number of implicit zeros, and per (column, block) the number of stored keys the block reads
+__global__ void k_csc_keys(const float* __restrict__ values, const int64_t* __restrict__ col_ptr, int64_t n, int c0,
+                           uint32_t* __restrict__ keys, int64_t ldk, int32_t* __restrict__ zeros,
+                           int32_t* __restrict__ cnt0, int row_blocks) {
+  const int j = blockIdx.y;
+  const int64_t p0 = col_ptr[c0 + j], nz = col_ptr[c0 + j + 1] - p0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nz; i += (int64_t)gridDim.x * blockDim.x)
+    keys[(int64_t)j * ldk + i] = f2key(values[p0 + i]);
+  if (blockIdx.x == 0) {
+    if (threadIdx.x == 0) zeros[j] = (int32_t)(n - nz);
+    for (int b = threadIdx.x; b < row_blocks; b += blockDim.x) {
+      const int64_t left = nz - (int64_t)b * kSelRows;
+      cnt0[(int64_t)j * row_blocks + b] = (int32_t)(left <= 0 ? 0 : (left < kSelRows ? left : kSelRows));
+    }
+  }
+}
+
+// the implicit zeros of each column join the counters of this pass (if their prefix is in A)
+__global__ void k_sel_zeros(int tc, int pbits, const int32_t* __restrict__ zeros, const SelMeta* __restrict__ meta,
+                            const uint32_t* __restrict__ pre, uint32_t* __restrict__ ghist) {
+  const int col = blockIdx.x * blockDim.x + threadIdx.x;
+  if (col >= tc || zeros[col] <= 0) return;
+  const uint32_t key0 = f2key(0.0f);
+  int e = -1;
+  if (!pbits) {
+    e = (int)(key0 >> 20);
+  } else {
+    const uint32_t kp = key0 >> (32 - pbits);
+    const int an = meta[col].an;
+    for (int i = 0; i < an; ++i)
+      if (pre[col * kSelMax + i] == kp) { e = i * kSelDigits + (int)((key0 >> (28 - pbits)) & 15u); break; }
+  }
+  if (e >= 0) ghist[(int64_t)col * kSelHist + e] += (uint32_t)zeros[col];
+}
+
+// bins of a CSC column tile: every row gets bin(0) of its column, then the stored values theirs
+__global__ void k_csc_zero_bins(int64_t n, int c0, int tc, int B, const float* __restrict__ cuts,
+                                const int32_t* __restrict__ nbins, uint8_t* __restrict__ bins, int64_t ld_bins) {
+  __shared__ uint8_t zb[kBinTC];
+  for (int j = threadIdx.x; j < tc; j += blockDim.x) {
+    const float* c = cuts + (int64_t)(c0 + j) * (B - 1);
+    const int nc = nbins[c0 + j] - 1;
+    int k = 0;
+    while (k < nc && c[k] <= 0.0f) ++k;
+    zb[j] = (uint8_t)k;
+  }
+  __syncthreads();
+  const int64_t total = n * tc;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = e / tc;
+    const int j = (int)(e - i * tc);
+    bins[i * ld_bins + c0 + j] = zb[j];
+  }
+}
+
+__global__ void __launch_bounds__(256)
+k_csc_apply(const float* __restrict__ values, const int32_t* __restrict__ row_idx, const int64_t* __restrict__ col_ptr,
+            int c0, int B, const float* __restrict__ cuts, const int32_t* __restrict__ nbins,
+            uint8_t* __restrict__ bins, int64_t ld_bins) {
+  __shared__ float c[256];
+  const int j = blockIdx.y;
+  for (int k = threadIdx.x; k < B - 1; k += blockDim.x) c[k] = cuts[(int64_t)(c0 + j) * (B - 1) + k];
+  __syncthreads();
+  const int ncut = nbins[c0 + j] - 1;
+  const int64_t p0 = col_ptr[c0 + j], p1 = col_ptr[c0 + j + 1];
+  for (int64_t p = p0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < p1; p += (int64_t)gridDim.x * blockDim.x) {
+    const float x = values[p];
+    int lo = 0;
+#pragma unroll
+    for (int st = 128; st > 0; st >>= 1)
+      if (lo + st <= ncut && c[lo + st - 1] <= x) lo += st;
+    bins[(int64_t)row_idx[p] * ld_bins + c0 + j] = (uint8_t)lo;
+  }
+}
+
+struct SelWs {
+  int64_t ldk;
+  unsigned row_blocks;
+  uint32_t *ka, *kb, *pre, *base, *ghist;
+  SelMeta* meta;
+  int32_t *cnt_a, *cnt_b, *cnt_0, *zeros;
+};
+
+// workspace: keys, compacted keys [tc][ldk] u32 | meta [tc] | prefixes, bases [tc][kSelMax] u32 |
+// counters [tc][kSelHist] u32 | kept-key counts 3 x [tc][row blocks] i32 | implicit zeros [tc] i32
+static size_t sel_ws_bytes(int64_t n, int32_t m) {
+  const int64_t tc = m < kBinTC ? m : kBinTC;
+  const int64_t rb = (n + kSelRows - 1) / kSelRows;
+  return (size_t)(2 * tc * ((n + 3) / 4 * 4) * 4 + tc * (int64_t)sizeof(SelMeta) + 2 * tc * kSelMax * 4 +
+                  tc * kSelHist * 4 + 3 * tc * rb * 4 + tc * 4 + 1024);
+}
+
+static SelWs sel_ws(void* ws, int64_t n, int32_t m) {
+  SelWs w;
+  const int64_t tcmax = m < kBinTC ? m : kBinTC;
+  w.ldk = (n + 3) / 4 * 4;                                 // 16-byte aligned key columns
+  w.row_blocks = (unsigned)((n + kSelRows - 1) / kSelRows);
+  w.ka = (uint32_t*)ws;
+  w.kb = w.ka + tcmax * w.ldk;
+  w.meta = (SelMeta*)(w.kb + tcmax * w.ldk);
+  w.pre = (uint32_t*)(w.meta + tcmax);
+  w.base = w.pre + tcmax * kSelMax;
+  w.ghist = w.base + tcmax * kSelMax;
+  w.cnt_a = (int32_t*)(w.ghist + tcmax * kSelHist);       // kept keys per (column, block)
+  w.cnt_b = w.cnt_a + tcmax * w.row_blocks;
+  w.cnt_0 = w.cnt_b + tcmax * w.row_blocks;               // CSC: stored keys per (column, block)
+  w.zeros = w.cnt_0 + tcmax * w.row_blocks;
+  return w;
+}
+
+// cuts and nbins of a column tile whose keys are in w.ka.  csc: w.cnt_0 / w.zeros describe the
+// stored keys and the implicit zeros of each column.
+static gbdtmo_status run_selection(Ctx* ctx, const SelWs& w, int64_t n, int tc, int B, bool csc, float* cuts, int32_t* nbins) {
+  GB_LAUNCH(k_sel_init, (unsigned)tc, 256, 0, tc, w.meta, w.pre, w.base, w.ghist);
+  // prefix bits before each pass: 0 (12-bit digit), then 12, 16, 20, 24, 28 (4-bit digits);
+  // from 16 bits on, the matched keys are compacted and only they are read by the next pass
+  const int pb[6] = {0, 12, 16, 20, 24, 28};
+  for (int k = 0; k < 6; ++k) {
+    const bool rd_c = pb[k] >= 20, wr_c = pb[k] >= 16 && pb[k] <= 24;
+    const uint32_t* kin = (pb[k] == 20 || pb[k] == 28) ? w.kb : w.ka;
+    uint32_t* kout = wr_c ? (pb[k] == 20 ? w.ka : w.kb) : nullptr;
+    const int32_t* cin = rd_c ? ((pb[k] == 24) ? w.cnt_b : w.cnt_a) : (csc ? w.cnt_0 : nullptr);
+    int32_t* cout = wr_c ? ((pb[k] == 20) ? w.cnt_b : w.cnt_a) : nullptr;
+    GB_LAUNCH(k_sel_count, dim3(w.row_blocks, (unsigned)tc), 256, 0, kin, cin, n, w.ldk, pb[k], w.meta, w.pre, w.ghist,
+              kout, cout);
+    if (csc) GB_LAUNCH(k_sel_zeros, (unsigned)((tc + 63) / 64), 64, 0, tc, pb[k], w.zeros, w.meta, w.pre, w.ghist);
+    GB_LAUNCH(k_sel_refine, (unsigned)tc, kSelMax, 0, n, B, (int)(pb[k] == 0), w.meta, w.pre, w.base, w.ghist);
+  }
+  GB_LAUNCH(k_sel_cuts, (unsigned)tc, 256, 0, n, B, w.meta, w.pre, w.base, cuts, nbins);
+  return GBDTMO_OK;
+}
+
 }  // namespace gbdtmo
 
 using namespace gbdtmo;
 
-// workspace: keys, compacted keys [tc][ldk] u32 | meta [tc] | prefixes, bases [tc][kSelMax] u32 | counters [tc][kSelHist] u32
 extern "C" size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B) {
   (void)B;
-  const int64_t tc = m < kBinTC ? m : kBinTC;
-  return (size_t)(2 * tc * ((n + 3) / 4 * 4) * 4 + tc * (int64_t)sizeof(SelMeta) + 2 * tc * kSelMax * 4 + tc * kSelHist * 4 +
-                  2 * tc * ((n + kSelRows - 1) / kSelRows) * 4 + 1024);
+  return sel_ws_bytes(n, m);
 }
 
 extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t B,
@@ -381,17 +513,7 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
   if (B > 256) { ctx->err = "gbdtmo_bin: B > 256 unsupported (bins are uint8)"; return GBDTMO_EUNSUPPORTED; }
   GB_CHECK_ARG(B >= 2, "B < 2");
   if (ws_bytes < gbdtmo_bin_workspace_bytes(n, m, B)) { ctx->err = "gbdtmo_bin: workspace too small"; return GBDTMO_ENOMEM; }
-  const int64_t tcmax = m < kBinTC ? m : kBinTC;
-  const int64_t ldk = (n + 3) / 4 * 4;                    // 16-byte aligned key columns
-  uint32_t* ka = (uint32_t*)ws;
-  uint32_t* kb = ka + tcmax * ldk;
-  SelMeta* meta = (SelMeta*)(kb + tcmax * ldk);
-  uint32_t* pre = (uint32_t*)(meta + tcmax);
-  uint32_t* base = pre + tcmax * kSelMax;
-  uint32_t* ghist = base + tcmax * kSelMax;
-  const unsigned row_blocks = (unsigned)((n + kSelRows - 1) / kSelRows);
-  int32_t* cnt_a = (int32_t*)(ghist + tcmax * kSelHist);    // kept keys per (column, block)
-  int32_t* cnt_b = cnt_a + tcmax * row_blocks;
+  const SelWs w = sel_ws(ws, n, m);
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(k_bin_apply, cudaFuncAttributeMaxDynamicSharedMemorySize, kBinTC * 255 * 4);
@@ -399,24 +521,49 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
   }
   for (int c0 = 0; c0 < m; c0 += kBinTC) {
     const int tc = (int)(m - c0 < kBinTC ? m - c0 : kBinTC);
-    GB_LAUNCH(k_bin_keys, dim3((unsigned)((n + 31) / 32), (unsigned)((tc + 31) / 32)), dim3(32, 8), 0, X, n, ld_x, c0, tc, ka, ldk);
-    GB_LAUNCH(k_sel_init, (unsigned)tc, 256, 0, tc, meta, pre, base, ghist);
-    // prefix bits before each pass: 0 (12-bit digit), then 12, 16, 20, 24, 28 (4-bit digits);
-    // from 16 bits on, the matched keys are compacted and only they are read by the next pass
-    const int pb[6] = {0, 12, 16, 20, 24, 28};
-    for (int k = 0; k < 6; ++k) {
-      const bool rd_c = pb[k] >= 20, wr_c = pb[k] >= 16 && pb[k] <= 24;
-      const uint32_t* kin = (pb[k] == 20 || pb[k] == 28) ? kb : ka;
-      uint32_t* kout = wr_c ? (pb[k] == 20 ? ka : kb) : nullptr;
-      const int32_t* cin = rd_c ? ((pb[k] == 24) ? cnt_b : cnt_a) : nullptr;
-      int32_t* cout = wr_c ? ((pb[k] == 20) ? cnt_b : cnt_a) : nullptr;
-      GB_LAUNCH(k_sel_count, dim3(row_blocks, (unsigned)tc), 256, 0, kin, cin, n, ldk, pb[k], meta, pre, ghist, kout,
-                cout);
-      GB_LAUNCH(k_sel_refine, (unsigned)tc, kSelMax, 0, n, B, (int)(pb[k] == 0), meta, pre, base, ghist);
+    GB_LAUNCH(k_bin_keys, dim3((unsigned)((n + 31) / 32), (unsigned)((tc + 31) / 32)), dim3(32, 8), 0, X, n, ld_x, c0,
+              tc, w.ka, w.ldk);
+    const gbdtmo_status st = run_selection(ctx, w, n, tc, B, false, cuts + (int64_t)c0 * (B - 1), nbins + c0);
+    if (st != GBDTMO_OK) return st;
+    GB_LAUNCH(k_bin_apply, ctx->num_sms * 2, kApplyThreads, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts,
+              nbins, bins, ld_bins);
+  }
+  return GBDTMO_OK;
+}
+
+extern "C" gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx c, const float* values, const int32_t* row_idx,
+                                        const int64_t* col_ptr, const int64_t* col_ptr_host, int64_t n, int32_t m,
+                                        int32_t B, uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
+                                        void* ws, size_t ws_bytes) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  GB_CHECK_ARG(col_ptr && col_ptr_host && bins && cuts && nbins && ws, "null pointer");
+  GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
+  GB_CHECK_ARG(n >= 1 && n < (int64_t(1) << 31) && m >= 1, "bad n or m");
+  GB_CHECK_ARG(ld_bins >= m, "bad leading dimension");
+  if (B > 256) { ctx->err = "gbdtmo_bin_csc: B > 256 unsupported (bins are uint8)"; return GBDTMO_EUNSUPPORTED; }
+  GB_CHECK_ARG(B >= 2, "B < 2");
+  GB_CHECK_ARG(col_ptr_host[0] == 0, "col_ptr[0] must be 0");
+  for (int32_t j = 0; j < m; ++j)
+    GB_CHECK_ARG(col_ptr_host[j + 1] >= col_ptr_host[j] && col_ptr_host[j + 1] - col_ptr_host[j] <= n,
+                 "col_ptr must be non-decreasing with at most n entries per column");
+  GB_CHECK_ARG(col_ptr_host[m] == 0 || (values && row_idx), "null values / row_idx");
+  if (ws_bytes < gbdtmo_bin_workspace_bytes(n, m, B)) { ctx->err = "gbdtmo_bin_csc: workspace too small"; return GBDTMO_ENOMEM; }
+  const SelWs w = sel_ws(ws, n, m);
+  for (int c0 = 0; c0 < m; c0 += kBinTC) {
+    const int tc = (int)(m - c0 < kBinTC ? m - c0 : kBinTC);
+    int64_t maxnz = 1;
+    for (int j = 0; j < tc; ++j) {
+      const int64_t nz = col_ptr_host[c0 + j + 1] - col_ptr_host[c0 + j];
+      maxnz = nz > maxnz ? nz : maxnz;
     }
-    GB_LAUNCH(k_sel_cuts, (unsigned)tc, 256, 0, n, B, meta, pre, base, cuts + (int64_t)c0 * (B - 1), nbins + c0);
-    GB_LAUNCH(k_bin_apply, ctx->num_sms * 2, kApplyThreads, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts, nbins, bins,
-              ld_bins);
+    const unsigned gx = (unsigned)((maxnz + 255) / 256 < 1024 ? (maxnz + 255) / 256 : 1024);
+    GB_LAUNCH(k_csc_keys, dim3(gx, (unsigned)tc), 256, 0, values, col_ptr, n, c0, w.ka, w.ldk, w.zeros, w.cnt_0,
+              (int)w.row_blocks);
+    const gbdtmo_status st = run_selection(ctx, w, n, tc, B, true, cuts + (int64_t)c0 * (B - 1), nbins + c0);
+    if (st != GBDTMO_OK) return st;
+    GB_LAUNCH(k_csc_zero_bins, ctx->num_sms * 4, 256, 0, n, c0, tc, B, cuts, nbins, bins, ld_bins);
+    GB_LAUNCH(k_csc_apply, dim3(gx, (unsigned)tc), 256, 0, values, row_idx, col_ptr, c0, B, cuts, nbins, bins, ld_bins);
   }
   return GBDTMO_OK;
 }

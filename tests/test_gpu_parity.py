@@ -107,6 +107,70 @@ def test_bin_selection_edge_cases(orc, pkg, ctx, n):
         np.testing.assert_array_equal(gb.T, bins)
 
 
+# ------------------------------------------------------------ CSC input
+
+def _csc_check(orc, pkg, ctx, X, B):
+    values, row_idx, col_ptr = orc.csc_from_dense(X)
+    n = X.shape[0]
+    ds = pkg.bin_features_csc(ctx, torch.from_numpy(values).to(DEV), torch.from_numpy(row_idx).to(DEV),
+                              torch.from_numpy(col_ptr), n, B)
+    torch.cuda.synchronize()
+    cuts, nbins, bins = orc.bin_matrix(X, B)
+    np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+    np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+    gb = ds.bins[: n * ds.ld_bins].view(n, ds.ld_bins)[:, : X.shape[1]].cpu().numpy()
+    np.testing.assert_array_equal(gb.T, bins)
+    return ds
+
+
+def test_bin_csc_paper_example(orc, pkg, ctx):
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "csc_example.json")))
+    for B in (2, 4, 256):
+        _csc_check(orc, pkg, ctx, np.array(g["dense"], np.float32), B)
+
+
+@pytest.mark.parametrize("n,density", [(1, 0.5), (7, 0.3), (5000, 0.19), (40001, 0.05), (40001, 0.9)])
+def test_bin_csc_equals_dense(orc, pkg, ctx, n, density):
+    rng = np.random.default_rng(n)
+    m = 70                                                           # two column tiles
+    X = np.where(rng.random((n, m)) < density, rng.normal(size=(n, m)), 0.0).astype(np.float32)
+    X[:, 3] = 0.0                                                    # empty column
+    X[:, 4] = rng.normal(size=n)                                     # fully dense column
+    X[:, 5] = np.where(rng.random(n) < density, -np.abs(rng.normal(size=n)), 0.0)   # zero is the maximum
+    X[:, 6] = np.where(rng.random(n) < density, rng.integers(1, 300, n), 0)         # few / many distinct
+    for B in (16, 256):
+        _csc_check(orc, pkg, ctx, X, B)
+
+
+def test_bin_csc_explicit_zeros(orc, pkg, ctx):
+    # stored 0.0 / -0.0 entries are ordinary values equal to the implicit zeros
+    rng = np.random.default_rng(11)
+    n, m = 3000, 9
+    X = np.where(rng.random((n, m)) < 0.3, rng.normal(size=(n, m)), 0.0).astype(np.float32)
+    vals, rows, ptr = [], [], [0]
+    for j in range(m):
+        keep = np.nonzero((X[:, j] != 0) | (rng.random(n) < 0.2))[0]     # some zeros stored explicitly
+        v = X[keep, j].copy()
+        v[(v == 0) & (rng.random(len(v)) < 0.5)] = -0.0
+        vals.append(v); rows.append(keep.astype(np.int32)); ptr.append(ptr[-1] + len(keep))
+    ds = pkg.bin_features_csc(ctx, torch.from_numpy(np.concatenate(vals)).to(DEV),
+                              torch.from_numpy(np.concatenate(rows)).to(DEV), torch.tensor(ptr, dtype=torch.int64), n, 256)
+    torch.cuda.synchronize()
+    cuts, nbins, bins = orc.bin_matrix(X, 256)
+    np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+    np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+    gb = ds.bins[: n * ds.ld_bins].view(n, ds.ld_bins)[:, :m].cpu().numpy()
+    np.testing.assert_array_equal(gb.T, bins)
+
+
+def test_bin_csc_mnist_shaped(orc, pkg, ctx):
+    w = CASES["C2s"]
+    X = gen.features_host(w)
+    _csc_check(orc, pkg, ctx, X, w.B)
+
+
 # ------------------------------------------------------------------------- gradients
 
 @pytest.mark.parametrize("case", ["C1", "C2s"])

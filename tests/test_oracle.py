@@ -67,6 +67,41 @@ def test_bin_mnist_shaped_column(orc):
     assert 0.79 < frac0 < 0.83
 
 
+# ------------------------------------------------------- CSC storage
+
+def _golden(name):
+    import json
+    import os
+    return json.load(open(os.path.join(os.path.dirname(__file__), "golden", name)))
+
+
+def test_csc_matches_paper_worked_example(orc):
+    # PAPER.md:181-201 prints the dense rows of x0..x4 and their CSC arrays (tests/golden/csc_example.json)
+    g = _golden("csc_example.json")
+    X = np.array(g["dense"], np.float32)
+    values, row_idx, col_ptr = orc.csc_from_dense(X)
+    assert values.tolist() == g["values"]
+    assert row_idx.tolist() == g["row_indices"]
+    assert col_ptr.tolist() == g["col_pointers"]
+    back = orc.dense_from_csc(np.array(g["values"]), np.array(g["row_indices"]), np.array(g["col_pointers"]), 5)
+    np.testing.assert_array_equal(back, X)
+
+
+def test_csc_round_trip_and_scipy(orc):
+    # independent library special case: scipy.sparse's CSC of the same matrix
+    import scipy.sparse as sp
+    rng = np.random.default_rng(3)
+    X = np.where(rng.random((300, 17)) < 0.8, 0.0, rng.normal(size=(300, 17))).astype(np.float32)
+    X[:, 5] = 0.0                                        # an empty column
+    values, row_idx, col_ptr = orc.csc_from_dense(X)
+    ref = sp.csc_matrix(X)
+    ref.sort_indices()
+    np.testing.assert_array_equal(col_ptr, ref.indptr)
+    np.testing.assert_array_equal(row_idx, ref.indices)
+    np.testing.assert_array_equal(values, ref.data)
+    np.testing.assert_array_equal(orc.dense_from_csc(values, row_idx, col_ptr, 300), X)
+
+
 # ------------------------------------------------------------------- gradients
 
 def _mse_loss(y, p):

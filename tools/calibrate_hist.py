@@ -41,8 +41,11 @@ def time_trees(ctx, ds, Y, w, thr, small=0, warm=2, timed=3):
 
 
 def main():
-    shapes = [gen.WORKLOADS["C2"], gen.WORKLOADS["C3"], gen.sweep(5), gen.sweep(10), gen.sweep(50),
-              gen.WORKLOADS["C5"].scaled(n=500_000, m=1024), gen.WORKLOADS["C1"]]
+    shapes = [gen.WORKLOADS["C2"], gen.WORKLOADS["C3"], gen.WORKLOADS["C4"], gen.sweep(5), gen.sweep(10),
+              gen.sweep(50), gen.WORKLOADS["C5"].scaled(n=500_000, m=1024), gen.WORKLOADS["C1"]]
+    only = sys.argv[1:]
+    if only:
+        shapes = [w for w in shapes if w.name.split("-")[0] in only]
     ctx = pkg.Context(0)
     entries = []
     for w in shapes:
@@ -55,7 +58,8 @@ def main():
         best = min(res, key=res.get)
         if res[best] > 0.98 * res[0]:          # noise guard: keep the default unless >= 2% faster
             best = 0
-        rs = {c: time_trees(ctx, ds, Y, w, best, c) for c in SMALL_CANDIDATES}
+        small_ok = w.d <= 32
+        rs = {c: time_trees(ctx, ds, Y, w, best, c) for c in (SMALL_CANDIDATES if small_ok else [0])}
         best_s = min(rs, key=rs.get)
         if rs[best_s] > 0.98 * rs[0]:
             best_s = 0
@@ -66,9 +70,13 @@ def main():
         print(json.dumps(entries[-1]), flush=True)
         del ds, Y
         torch.cuda.empty_cache()
+    path = os.path.join(ROOT, "paper_conf_icpp_liupw25_b200", "hist_variant_table.json")
+    if only and os.path.exists(path):                    # partial run: merge into the existing table
+        old = json.load(open(path)).get("entries", [])
+        names = {e["workload"] for e in entries}
+        entries = [e for e in old if e["workload"] not in names] + entries
     out = {"measured": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
            "device": torch.cuda.get_device_name(0), "candidates": CANDIDATES, "entries": entries}
-    path = os.path.join(ROOT, "paper_conf_icpp_liupw25_b200", "hist_variant_table.json")
     json.dump(out, open(path, "w"), indent=1)
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     json.dump(out, open(os.path.join(ROOT, "gpurun_out", "hist_variant_table.json"), "w"), indent=1)

@@ -20,5 +20,9 @@ timeout 1500 ncu --set full --clock-control none --import-source on -k regex:k_h
     -o $out/${tag}_prof_hist_c5 python tools/prof_run.py C5 1 > $out/${tag}_ncu_hist.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_find_split -s 3 -c 3 \
     -o $out/${tag}_prof_fs_c5 python tools/prof_run.py C5 1 > $out/${tag}_ncu_fs.log 2>&1
-# 4. micro-benchmarks of the on-chip accumulation pipes
+# 4. binning (once per dataset): warm timing and its launch list on C5
+timeout 300 python tools/bin_probe.py C5 > $out/${tag}_bin_probe_c5.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+    --log-file $out/${tag}_launches_bin_c5.csv python tools/bin_probe.py C5 > $out/${tag}_ncu_bin.log 2>&1
+# 5. micro-benchmarks of the on-chip accumulation pipes
 ./tools/microbench/atom_bench > $out/${tag}_atom_bench.txt 2>&1 || true

@@ -39,7 +39,7 @@ def launch_summary(csv_path, txt_path):
             continue
         agg[name][0] += 1
         agg[name][1] += v
-    setup = ("radix", "bin_", "gen_", "k_default_bins", "at::")
+    setup = ("radix", "bin_", "k_sel_", "k_csc_", "gen_", "k_default_bins", "at::")
     tree = {k: v for k, v in agg.items() if not any(s in k for s in setup)}
     tot_tree = sum(v[1] for v in tree.values())
     with open(txt_path, "w") as f:
@@ -97,6 +97,14 @@ def main():
                                "dram_bytes_per_launch": tot / cnt, "launches": cnt,
                                "source": f"profiles/{tag}_ncu_hist_c5.txt (ncu --set full, one tree)"},
                               open(os.path.join(PROF, "hist_traffic.json"), "w"), indent=1)
+    bp = os.path.join(OUT, f"{tag}_bin_probe_c5.log")
+    if os.path.exists(bp):
+        j = last_json(bp)
+        if j:
+            json.dump(j, open(os.path.join(PROF, f"{tag}_bin_probe_c5.json"), "w"), indent=1)
+    bl = os.path.join(OUT, f"{tag}_launches_bin_c5.csv")
+    if os.path.exists(bl):
+        launch_summary(bl, os.path.join(PROF, f"{tag}_launches_bin_c5_summary.txt"))
     ab = os.path.join(OUT, f"{tag}_atom_bench.txt")
     if os.path.exists(ab):
         subprocess.run(["cp", ab, os.path.join(PROF, f"{tag}_microbench_atomics.txt")])

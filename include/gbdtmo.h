@@ -105,8 +105,12 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *   GBDTMO_OPT_SMALL_MAX_ROWS: fused small-node path — when both children of a split have at most
  *     this many rows they are marked SMALL: built from their rows and searched in shared memory by
  *     gbdtmo_search_small, never materialised and not derived by subtraction (reading R27);
- *     0 (default) = off.  Requires d <= 32 and a feature tile that fits shared memory. */
-enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2 };
+ *     0 (default) = off.  Requires d <= 32 and a feature tile that fits shared memory.
+ *   GBDTMO_OPT_HIST_KERNEL: shared-memory histogram lane mapping — 0 (default): channel tiles of
+ *     K = 4/8/16 with 32/K rows per instruction; 1: "diagonal" channel tiles of 4, eight rows per
+ *     instruction each adding to a different slot, conflict-free for any channel count (DESIGN.md
+ *     §7).  Same results; chosen per workload shape by measurement.  Not used with default bins. */
+enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3 };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Number of kernels this context has launched so far (for launch accounting). */
 int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);

@@ -27,7 +27,7 @@ SYMBOLS = (
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc",
 )
-OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS = 1, 2
+OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL = 1, 2, 3
 
 
 class GbdtmoError(RuntimeError):

@@ -136,7 +136,7 @@ class Booster:
     def __init__(self, ctx: Context, ds: Dataset, y: torch.Tensor, params: Params,
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
-                 small_max_rows: Optional[int] = None):
+                 small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None):
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
         # histogram variant selection: nodes with <= gmem_max_rows
         # rows use the global-atomic variant; None = the measured table for this channel count
@@ -144,6 +144,9 @@ class Booster:
         self.gmem_max_rows = variant_threshold(V, ds.m, n=ds.n) if gmem_max_rows is None else int(gmem_max_rows)
         self.small_max_rows = variant_threshold(V, ds.m, "small_max_rows", n=ds.n) if small_max_rows is None \
             else int(small_max_rows)
+        # shared-memory lane mapping: 0 row-pair tiles, 1 diagonal K = 4 tiles (measured per shape)
+        self.hist_kernel = variant_threshold(V, ds.m, "hist_kernel", n=ds.n) if hist_kernel is None \
+            else int(hist_kernel)
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
@@ -214,6 +217,7 @@ class Booster:
         ctx.gbdtmo_set_stream(torch.cuda.current_stream(self.device).cuda_stream)
         ctx.gbdtmo_set_option(_abi.OPT_GMEM_MAX_ROWS, self.gmem_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
+        ctx.gbdtmo_set_option(_abi.OPT_HIST_KERNEL, self.hist_kernel)
 
     def _tree(self, time_hist: bool = False):
         ctx, p = self.ctx, self.p

@@ -22,6 +22,7 @@ struct Ctx {
   int64_t launches = 0;
   int64_t gmem_max_rows = 0;   // GBDTMO_OPT_GMEM_MAX_ROWS: BUILD nodes with <= rows use the global-atomic variant
   int64_t small_max_rows = 0;  // GBDTMO_OPT_SMALL_MAX_ROWS: nodes whose parent's children both fit -> fused path
+  int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16) variant, 1 diagonal (K = 4) variant
   std::string err;
 };
 
@@ -212,6 +213,11 @@ inline const char* check_problem(const gbdtmo_problem* p) {
   if (p->ld_bins < p->m || p->ld_bins % 8 != 0) return "ld_bins must be >= m and a multiple of 8";
   return nullptr;
 }
+
+// The diagonal shared-memory histogram variant (hist_diag.cu).
+HistCfg hist_config_diag(const gbdtmo_problem& p);
+gbdtmo_status launch_hist_diag(Ctx* ctx, const gbdtmo_problem& p, const uint8_t* bins, const int32_t* q,
+                               const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt);
 
 // Histogram work items wanted per level -> chunks per build level (grad.cu).
 int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p);

@@ -337,7 +337,9 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
   const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
   const int use_rows = level > 0;
   gbdtmo_status st;
-  switch (hc.K) {
+  if (ctx->hist_kernel == 1 && !dflt) {
+    st = launch_hist_diag(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
+  } else switch (hc.K) {
     case 4: st = launch_hist<4>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
     case 8: st = launch_hist<8>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
     default: st = launch_hist<16>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;

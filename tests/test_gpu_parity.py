@@ -202,8 +202,8 @@ def test_grad_matches_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------------ histograms
 
-@pytest.mark.parametrize("case", ["C1", "C3s", "C5s", "C2s", "C4s"])
-def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
+@pytest.mark.parametrize("case,hk", [(c, k) for k in (0, 1) for c in ("C1", "C3s", "C5s", "C2s", "C4s")])
+def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
     """Every level's histograms (built and derived by subtraction) vs the oracle's direct
     per-node histograms over the oracle's node rows; exact on tree-1 dyadic MSE inputs."""
     w = CASES[case]
@@ -214,8 +214,8 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
     rows = node_rows(bins, ref["state"][0], ref["feat"][0], ref["bin"][0], w.n)
     g, h = orc.grad(w.loss, Y.astype(np.float64), np.zeros(Y.shape))
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1), sparse_default=True,
-                    gmem_max_rows=0, small_max_rows=0)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w, T=1), sparse_default=(hk == 0),
+                    gmem_max_rows=0, small_max_rows=0, hist_kernel=hk)
     b._apply_options()
     ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
     sc = None
@@ -254,13 +254,15 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------- whole trees
 
-@pytest.mark.parametrize("case,sparse,gmem,small", [
-    ("C1", False, 0, 0), ("C2s", False, 0, 0), ("C2s", True, 0, 0), ("C3s", False, 0, 0), ("C4s", False, 0, 0),
-    ("C5s", False, 0, 0), ("S300s", False, 0, 0),
-    ("C3s", False, 1 << 30, 0), ("C2s", True, 3000, 0), ("C5s", False, 5000, 0),            # global-atomic variant
-    ("C1", False, 0, 2000), ("C2s", False, 0, 4000), ("C2s", True, 256, 2500),               # sort-and-segment small nodes
-    ("C3s", False, 0, 9000), ("C5s", False, 0, 6000)])
-def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, small):
+@pytest.mark.parametrize("case,sparse,gmem,small,hk", [
+    ("C1", False, 0, 0, 0), ("C2s", False, 0, 0, 0), ("C2s", True, 0, 0, 0), ("C3s", False, 0, 0, 0),
+    ("C4s", False, 0, 0, 0), ("C5s", False, 0, 0, 0), ("S300s", False, 0, 0, 0),
+    ("C3s", False, 1 << 30, 0, 0), ("C2s", True, 3000, 0, 0), ("C5s", False, 5000, 0, 0),   # global-atomic variant
+    ("C1", False, 0, 2000, 0), ("C2s", False, 0, 4000, 0), ("C2s", True, 256, 2500, 0),     # sort-and-segment small nodes
+    ("C3s", False, 0, 9000, 0), ("C5s", False, 0, 6000, 0),
+    ("C1", False, 0, 0, 1), ("C2s", False, 0, 0, 1), ("C3s", False, 0, 0, 1), ("C4s", False, 0, 0, 1),  # diagonal
+    ("C5s", False, 0, 0, 1), ("S300s", False, 0, 0, 1), ("C2s", False, 3000, 128, 1)])
+def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, small, hk):
     w = CASES[case]
     X, Y = _inputs(w)
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
@@ -268,7 +270,7 @@ def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, smal
                     lr=w.lr, min_node=w.min_node)
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
     b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), sparse_default=sparse, gmem_max_rows=gmem,
-                    small_max_rows=small)
+                    small_max_rows=small, hist_kernel=hk)
     assert (b.dflt is not None) == (sparse and w.index == 2)     # only the MNIST-shaped data has dominant bins
     b.fit()
     torch.cuda.synchronize()

@@ -109,7 +109,9 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *   GBDTMO_OPT_HIST_KERNEL: shared-memory histogram lane mapping — 0 (default): channel tiles of
  *     K = 4/8/16 with 32/K rows per instruction; 1: "diagonal" channel tiles of 4, eight rows per
  *     instruction each adding to a different slot, conflict-free for any channel count (DESIGN.md
- *     §7).  Same results; chosen per workload shape by measurement.  Not used with default bins. */
+ *     §7); 2: row-pair tiles whose bin windows are staged in shared memory by TMA gather4
+ *     (measured slower, kept as the recorded alternative).  Same results; chosen per workload
+ *     shape by measurement.  1 and 2 are not used with default bins. */
 enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3 };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Number of kernels this context has launched so far (for launch accounting). */
@@ -200,6 +202,24 @@ gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* 
 gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
                                 const uint8_t* bins, const int32_t* dflt, const int32_t* q, void* state,
                                 int64_t* hist, int32_t* cnt);
+
+/* Tile-packed bins for the histogram kernel (DESIGN.md §7 "Packed bins"; the B200 form of the
+ * paper's "bin packing").  The shared-memory histogram kernel works on tiles of k
+ * features (k from the problem's shape, at most 8 for a packed layout); with the row-major
+ * matrix every row of a tile is its own cache line, so a warp's 32 gathered rows cost 32-64 L1
+ * wavefronts per load.  The packed copy stores each tile's bins contiguously per row:
+ *   packed uint8 [n_tiles][n][8]:  packed[(t * n + i) * 8 + j] = bins[i * ld + k t + j] (j < k),
+ *                                  0 for j >= k or k t + j >= m,
+ * so adjacent rows are adjacent 8-byte words.  gbdtmo_packed_bins_bytes: bytes of `packed`, 0 when
+ * the problem's tiles are wider than 8 features (then use gbdtmo_build_hist).  The caller owns
+ * `packed`; gbdtmo_pack_bins fills it from `bins` (once per dataset and problem shape).
+ * gbdtmo_build_hist_packed = gbdtmo_build_hist reading the tile bins from `packed` (and `bins`
+ * for the global-atomic small-node variant); identical results. */
+size_t gbdtmo_packed_bins_bytes(const gbdtmo_problem* p);
+gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx ctx, const gbdtmo_problem* p, const uint8_t* bins, uint8_t* packed);
+gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                       const uint8_t* bins, const uint8_t* packed, const int32_t* dflt,
+                                       const int32_t* q, void* state, int64_t* hist, int32_t* cnt);
 
 /* ------------------------------------- (a)4 subtraction + (a)5 split search */
 

@@ -25,7 +25,8 @@ SYMBOLS = (
     "gbdtmo_hist_bytes", "gbdtmo_xchg_count", "gbdtmo_bin", "gbdtmo_grad", "gbdtmo_build_hist",
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
-    "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc",
+    "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
+    "gbdtmo_build_hist_packed",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL = 1, 2, 3
 
@@ -75,6 +76,9 @@ def lib():
             "gbdtmo_grad": ([P, PP, P, P, P, P, P], C.c_int),
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_build_hist_packed": ([P, PP, i32, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_packed_bins_bytes": ([PP], sz),
+            "gbdtmo_pack_bins": ([P, PP, P, P], C.c_int),
             "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_search_small": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
@@ -188,6 +192,18 @@ class Context:
     def gbdtmo_build_hist(self, p, level, bins, dflt, q, state, hist, cnt):
         self._check(lib().gbdtmo_build_hist(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(q),
                                             _ptr(state), _ptr(hist), _ptr(cnt)), "gbdtmo_build_hist")
+
+    def gbdtmo_build_hist_packed(self, p, level, bins, packed, dflt, q, state, hist, cnt):
+        self._check(lib().gbdtmo_build_hist_packed(self._h, C.byref(p), level, _ptr(bins), _ptr(packed), _ptr(dflt),
+                                                   _ptr(q), _ptr(state), _ptr(hist), _ptr(cnt)),
+                    "gbdtmo_build_hist_packed")
+
+    @staticmethod
+    def gbdtmo_packed_bins_bytes(p) -> int:
+        return int(lib().gbdtmo_packed_bins_bytes(C.byref(p)))
+
+    def gbdtmo_pack_bins(self, p, bins, packed):
+        self._check(lib().gbdtmo_pack_bins(self._h, C.byref(p), _ptr(bins), _ptr(packed)), "gbdtmo_pack_bins")
 
     def gbdtmo_find_split(self, p, level, nbins, dflt, scales, state, hist, cnt, parent_hist, parent_cnt, keys):
         self._check(lib().gbdtmo_find_split(self._h, C.byref(p), level, _ptr(nbins), _ptr(dflt), _ptr(scales),

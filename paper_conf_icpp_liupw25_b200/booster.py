@@ -136,7 +136,8 @@ class Booster:
     def __init__(self, ctx: Context, ds: Dataset, y: torch.Tensor, params: Params,
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
-                 small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None):
+                 small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
+                 packed_bins: Optional[bool] = None):
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
         # histogram variant selection: nodes with <= gmem_max_rows
         # rows use the global-atomic variant; None = the measured table for this channel count
@@ -175,6 +176,16 @@ class Booster:
             self.cnt[lvl % 2] = torch.empty(cb // 4, dtype=torch.int32, device=dev)
         if self.hist[1] is None:
             self.hist[1], self.cnt[1] = self.hist[0], self.cnt[0]
+        # tile-packed bins for the row-pair histogram kernel (gbdtmo_pack_bins):
+        # default on wherever the shape allows it and that kernel is selected
+        nb = ctx.gbdtmo_packed_bins_bytes(self.p)
+        use_packed = (nb > 0 and self.hist_kernel == 0) if packed_bins is None else bool(packed_bins)
+        self.packed = None
+        if use_packed:
+            assert nb > 0, "this problem shape has no packed bin layout"
+            self.packed = torch.empty(nb, dtype=torch.uint8, device=dev)
+            ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
+            ctx.gbdtmo_pack_bins(self.p, ds.bins, self.packed)
         self.keys = torch.zeros(1 << max(D - 1, 0), dtype=torch.int64, device=dev)
         self.xchg = torch.zeros(ctx.gbdtmo_xchg_count(self.p), dtype=torch.int64, device=dev)
         NH = (1 << (D + 1)) - 1
@@ -194,7 +205,11 @@ class Booster:
         if time_hist:
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-        ctx.gbdtmo_build_hist(p, lvl, self.ds.bins, self.dflt, self.q, self.state, self.hist[cur], self.cnt[cur])
+        if self.packed is not None:
+            ctx.gbdtmo_build_hist_packed(p, lvl, self.ds.bins, self.packed, self.dflt, self.q, self.state,
+                                         self.hist[cur], self.cnt[cur])
+        else:
+            ctx.gbdtmo_build_hist(p, lvl, self.ds.bins, self.dflt, self.q, self.state, self.hist[cur], self.cnt[cur])
         if time_hist:
             e1.record()
             self.hist_events.append((e0, e1))

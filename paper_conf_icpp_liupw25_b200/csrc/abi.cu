@@ -48,7 +48,7 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
     case GBDTMO_OPT_GMEM_MAX_ROWS: ctx->gmem_max_rows = value; return GBDTMO_OK;
     case GBDTMO_OPT_SMALL_MAX_ROWS: ctx->small_max_rows = value; return GBDTMO_OK;
     case GBDTMO_OPT_HIST_KERNEL:
-      if (value != 0 && value != 1) { ctx->err = "gbdtmo_set_option: HIST_KERNEL must be 0 or 1"; return GBDTMO_EINVAL; }
+      if (value < 0 || value > 2) { ctx->err = "gbdtmo_set_option: HIST_KERNEL must be 0, 1 or 2"; return GBDTMO_EINVAL; }
       ctx->hist_kernel = value;
       return GBDTMO_OK;
     default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;

@@ -22,7 +22,7 @@ struct Ctx {
   int64_t launches = 0;
   int64_t gmem_max_rows = 0;   // GBDTMO_OPT_GMEM_MAX_ROWS: BUILD nodes with <= rows use the global-atomic variant
   int64_t small_max_rows = 0;  // GBDTMO_OPT_SMALL_MAX_ROWS: nodes whose parent's children both fit -> fused path
-  int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16) variant, 1 diagonal (K = 4) variant
+  int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16), 1 diagonal (K = 4), 2 TMA-staged row-pair
   std::string err;
 };
 
@@ -90,26 +90,32 @@ struct HistCfg {
   int smem;   // bytes of dynamic shared memory
 };
 
+__host__ __device__ inline int hist_cnt_words(int K, int k, int B) { return k * B; }   // counts[k][B]
+
 __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   HistCfg c;
   int V = channels(p);
   c.K = V <= 4 ? 4 : V <= 8 ? 8 : 16;   // K = 32 halves the atomics per loaded row (measured slower)
   c.n_ct = (V + c.K - 1) / c.K;
-  int per_feature = p.B * (2 * c.K + 1) * 4;
+  const int limbs_per_feature = p.B * 2 * c.K * 4;
   // compile-time tile widths the kernel is instantiated for; each needs a per-warp scratch of
   // 32 rows x ceil(k/8) 8-byte bin words
   const int allowed[9] = {24, 16, 12, 8, 6, 4, 3, 2, 1};
   int k = 1;
   for (int i = 0; i < 9; ++i) {
     const int kk = allowed[i];
-    const int need = kk * per_feature + kHistWarps * 32 * 8 * ((kk + 7) / 8);
+    const int need = kk * limbs_per_feature + 4 * hist_cnt_words(c.K, kk, p.B) + kHistWarps * 32 * 8 * ((kk + 7) / 8);
     if (kk <= p.m && need <= kHistSmemBudget) { k = kk; break; }
   }
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
-  c.smem = k * per_feature + kHistWarps * 32 * 8 * ((k + 7) / 8);
+  c.smem = k * limbs_per_feature + 4 * hist_cnt_words(c.K, k, p.B) + kHistWarps * 32 * 8 * ((k + 7) / 8);
   return c;
 }
+
+// Tile-packed bins (gbdtmo_pack_bins): uint8 [n_ft][n][8], slot (t, i) = bins of features
+// [k t, k t + k) of row i, zero padded; only for tiles of <= 8 features.
+__host__ __device__ inline bool hist_packable(const gbdtmo_problem& p) { return hist_config(p).k <= 8; }
 
 // ------------------------------------------------------------- state layout
 
@@ -218,6 +224,11 @@ inline const char* check_problem(const gbdtmo_problem* p) {
 HistCfg hist_config_diag(const gbdtmo_problem& p);
 gbdtmo_status launch_hist_diag(Ctx* ctx, const gbdtmo_problem& p, const uint8_t* bins, const int32_t* q,
                                const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt);
+// The TMA-staged shared-memory histogram variant (hist_tma.cu).
+bool hist_tma_supported(const gbdtmo_problem& p, const uint8_t* bins);
+HistCfg hist_config_tma(const gbdtmo_problem& p, int max_smem);
+gbdtmo_status launch_hist_tma(Ctx* ctx, const gbdtmo_problem& p, const uint8_t* bins, const int32_t* q,
+                              const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt);
 
 // Histogram work items wanted per level -> chunks per build level (grad.cu).
 int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p);

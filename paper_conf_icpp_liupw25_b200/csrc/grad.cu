@@ -151,7 +151,9 @@ __global__ void k_root_plan(gbdtmo_problem p, State s, int target_chunks, int64_
 }
 
 int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p) {
-  HistCfg hc = ctx->hist_kernel == 1 ? hist_config_diag(p) : hist_config(p);
+  HistCfg hc = ctx->hist_kernel == 1 ? hist_config_diag(p)
+               : (ctx->hist_kernel == 2 && hist_tma_supported(p, nullptr)) ? hist_config_tma(p, ctx->max_smem_optin)
+                                                                          : hist_config(p);
   int64_t tiles = (int64_t)hc.n_ft * hc.n_ct;
   int64_t want = 4LL * ctx->num_sms;
   int64_t t = (want + tiles - 1) / tiles;

@@ -14,7 +14,15 @@
 //    one feature, all on distinct banks (lo/hi limbs of alternating rows are swapped);
 //  - each lane loads its row's q once and an 8-byte-aligned window (<= 32 bytes) of the row's
 //    bins once, then walks the tile's k features (the paper's "bin packing", PAPER.md:239,
-//    becomes one vector load of up to 32 bin ids).
+//    becomes one vector load of up to 32 bin ids);
+//  - with tile-packed bins (gbdtmo_pack_bins: [tile][row][8 bytes]) that window is one aligned
+//    8-byte load from a plane holding only this tile's bins: consecutive rows are adjacent, so
+//    a warp's 32 rows touch 2-32 cache lines instead of 32-64 (ncu: the gathered window loads
+//    were ~18% of the L1 data-pipe wavefronts, the pipe this kernel saturated);
+//  - the inner loop is kept to PRMT + 2 IMAD + 2 ATOMS per (row pair, feature): rows past the
+//    end of the item carry q = 0 and features past m sit in shared-memory slots that are never
+//    flushed, so neither needs a test; the two limbs come from one PRMT each with per-lane
+//    selectors; q is loaded one sub-batch ahead of use.
 #include "common.cuh"
 #include "hist_common.cuh"
 
@@ -30,10 +38,10 @@ namespace gbdtmo {
 // shifts it, counts it (CNT) and parks the bins in the scratch; then the K groups of
 // 32/K rows are accumulated, lanes (row, channel) reading their bins back with one LDS and
 // their q value from a batch-wide prefetch.
-template <int K, int KF, bool SKIP>
+template <int K, int KF, bool SKIP, bool PACKED>
 __global__ void __launch_bounds__(kHistThreads, 1)
-k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ dflt,
-            const int32_t* __restrict__ q,
+k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const uint8_t* __restrict__ packed,
+            const int32_t* __restrict__ dflt, const int32_t* __restrict__ q,
             const int32_t* __restrict__ rows, int use_rows, State s,
             int64_t* __restrict__ hist, int32_t* __restrict__ cnt) {
   extern __shared__ __align__(16) uint32_t sm[];
@@ -48,7 +56,8 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #endif
   constexpr int SB = G < GBDTMO_HIST_SB ? G : GBDTMO_HIST_SB;   // groups per q-prefetch sub-batch
   constexpr int RS = KF * 2 * K;               // limb words per bin
-  constexpr int NW = HistRow<KF>::NW, SW = HistRow<KF>::SW;
+  constexpr int NW = PACKED ? 1 : HistRow<KF>::NW, SW = PACKED ? 1 : HistRow<KF>::SW;
+  static_assert(!PACKED || KF <= 8, "packed tiles hold <= 8 features");
   const int V = channels(p), B = p.B, m = p.m;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
   const int ri = lane / K, c = lane % K;
@@ -63,6 +72,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   const uint32_t aA = sbase + 4u * slotA, aB = sbase + 4u * slotB;
   const uint32_t acnt = sbase + 4u * limb_words;
   const int64_t ld = p.ld_bins;
+  // limb selectors for PRMT(q, sel, 0): lo = bytes 0-1 zero-extended (0x4410), hi = bytes 2-3
+  // sign-extended (0xBB32); even rows add (lo, hi) at (slotA, slotB), odd rows (hi, lo)
+  const uint32_t selA = (ri & 1) ? 0xBB32u : 0x4410u, selB = (ri & 1) ? 0x4410u : 0xBB32u;
 
   for (;;) {
     if (threadIdx.x == 0) sh_item = atomicAdd(&s.misc[MISC_WORK_COUNTER], 1);
@@ -87,16 +99,18 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     __syncthreads();
 
     const int beg = ch.y, end = ch.z;
-    const int o = f0 & 7;
-    const uint8_t* bbase = bins + (f0 & ~7);
+    const int o = PACKED ? 0 : f0 & 7;
+    const uint8_t* bbase = PACKED ? packed + (int64_t)ft * p.n * 8 : bins + (f0 & ~7);
+    const int64_t rstride = PACKED ? 8 : ld;
     const bool chan_on = (c0 + c) < V;
     const int32_t* qc = q + c0 + c;
-    // cross-batch pipeline: row ids two batches ahead, bin windows one batch ahead
+    // cross-batch pipeline: row ids two batches ahead, bin windows one batch ahead, q one
+    // sub-batch ahead
     const int bstep = nwarps * 32;
     auto load_rid = [&](int pos) -> int { return pos < end ? (use_rows ? __ldg(&rows[pos]) : pos) : -1; };
     auto load_win = [&](int rr, uint64_t (&w)[NW]) {
       if (rr >= 0) {
-        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)rr * ld);
+        const uint64_t* wp = reinterpret_cast<const uint64_t*>(bbase + (int64_t)rr * rstride);
 #pragma unroll
         for (int i = 0; i < NW; ++i) w[i] = __ldg(wp + i);
       } else {
@@ -104,27 +118,42 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         for (int i = 0; i < NW; ++i) w[i] = 0;
       }
     };
+    auto load_q = [&](int rid, int t0, int (&qv)[SB]) {
+#pragma unroll
+      for (int t = 0; t < SB; ++t) {
+        const int rr = __shfl_sync(0xffffffffu, rid, (t0 + t) * RPI + ri);
+        qv[t] = (rr >= 0 && chan_on) ? __ldg(qc + (int64_t)rr * V) : 0;
+      }
+    };
     int r_cur = load_rid(beg + warp * 32 + lane);
     int r_nxt = load_rid(beg + warp * 32 + bstep + lane);
     uint64_t w_cur[NW];
     load_win(r_cur, w_cur);
+    int qv[SB];
+    load_q(r_cur, 0, qv);
     for (int b0 = beg + warp * 32; b0 < end; b0 += bstep) {
-      // ---- prefetch for the next batches
       const int r_nn = load_rid(b0 + 2 * bstep + lane);
       uint64_t w_nxt[NW];
       load_win(r_nxt, w_nxt);
-      // ---- phase 1: lane l owns row b0 + l
+      // ---- phase 1: lane l owns row b0 + l (invalid rows: window 0, q 0, not counted)
       const int r = r_cur;
       uint64_t sw[SW];
 #pragma unroll
       for (int i = 0; i < SW; ++i) sw[i] = 0;
       if (r >= 0) {
         shift_window<NW, SW>(w_cur, o, sw);
+        if (!PACKED && kk < KF) {                // last tile: bytes past feature m-1 -> bin 0
+#pragma unroll
+          for (int i = 0; i < SW; ++i) {
+            const int keep = kk - 8 * i;           // bytes of word i that hold features < m
+            sw[i] = keep >= 8 ? sw[i] : keep <= 0 ? 0ull : (sw[i] & ((1ull << (8 * keep)) - 1));
+          }
+        }
         if (do_cnt && !GBDTMO_HIST_NOCOUNT) {
 #pragma unroll
-          for (int j = 0; j < KF; ++j) {
+          for (int j = 0; j < KF; ++j) {         // features j >= kk land in slots never flushed
             const uint32_t bin = byte_of<SW>(sw, j);
-            if (j < kk && (!SKIP || (int)bin != dfl[j])) red_shared_add(acnt + 4u * (j * B + bin), 1u);  // counts[j][b]
+            if (!SKIP || (int)bin != dfl[j]) red_shared_add(acnt + 4u * (j * B + bin), 1u);  // counts[j][b]
           }
         }
       }
@@ -134,43 +163,28 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       // ---- phase 2: groups of RPI rows x K channels
 #pragma unroll
       for (int t0 = 0; t0 < G; t0 += SB) {
-        int qv[SB];
-#pragma unroll
-        for (int t = 0; t < SB; ++t) {
-          const int rr = __shfl_sync(0xffffffffu, r, (t0 + t) * RPI + ri);
-          qv[t] = (rr >= 0 && chan_on) ? __ldg(qc + (int64_t)rr * V) : 0;
-        }
+        int qn[SB];
+        if (t0 + SB < G) load_q(r, t0 + SB, qn);
+        else load_q(r_nxt, 0, qn);
 #pragma unroll
         for (int t = 0; t < SB; ++t) {
           const int i = (t0 + t) * RPI + ri;
-          if (b0 + i < end) {
-            uint64_t bw[SW];
+          uint64_t bw[SW];
 #pragma unroll
-            for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
-            const uint32_t lo = (uint32_t)qv[t] & 0xFFFFu;
-            const uint32_t hi = (uint32_t)(qv[t] >> 16);       // arithmetic shift, two's complement
-            const uint32_t va = (ri & 1) ? hi : lo, vb = (ri & 1) ? lo : hi;
-            if (kk == KF) {
+          for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
+          const uint32_t va = prmt_sx((uint32_t)qv[t], selA);
+          const uint32_t vb = prmt_sx((uint32_t)qv[t], selB);
 #pragma unroll
-              for (int j = 0; j < KF; ++j) {
-                const uint32_t bin = byte_of<SW>(bw, j);
-                if (!SKIP || (int)bin != dfl[j]) {
-                  red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-                  red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
-                }
-              }
-            } else {
-#pragma unroll
-              for (int j = 0; j < KF; ++j) {
-                const uint32_t bin = byte_of<SW>(bw, j);
-                if (j < kk && (!SKIP || (int)bin != dfl[j])) {
-                  red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-                  red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
-                }
-              }
+          for (int j = 0; j < KF; ++j) {
+            const uint32_t bin = byte_of<SW>(bw, j);
+            if (!SKIP || (int)bin != dfl[j]) {
+              red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+              red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
             }
           }
         }
+#pragma unroll
+        for (int t = 0; t < SB; ++t) qv[t] = qn[t];
       }
       __syncwarp();
       r_cur = r_nxt;
@@ -274,44 +288,96 @@ __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __re
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += stride) cb[i] = 0;
 }
 
-template <int K, int KF, bool SKIP>
+template <int K, int KF, bool SKIP, bool PACKED>
 static gbdtmo_status launch_hist_kfs(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
-                                     const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows,
-                                     const State& s, int64_t* hist, int32_t* cnt) {
+                                     const uint8_t* packed, const int32_t* dflt, const int32_t* q,
+                                     const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
   static bool attr_done = false;
   if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_smem<K, KF, SKIP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_hist_smem<K, KF, SKIP, PACKED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          ctx->max_smem_optin - 1024);
     attr_done = true;
   }
-  GB_LAUNCH((k_hist_smem<K, KF, SKIP>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, dflt, q, rows, use_rows, s,
-            hist, cnt);
+  GB_LAUNCH((k_hist_smem<K, KF, SKIP, PACKED>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, packed, dflt, q,
+            rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
 }
 
 template <int K, int KF>
 static gbdtmo_status launch_hist_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
-                                    const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows,
-                                    const State& s, int64_t* hist, int32_t* cnt) {
-  if (dflt) return launch_hist_kfs<K, KF, true>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-  return launch_hist_kfs<K, KF, false>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+                                    const uint8_t* packed, const int32_t* dflt, const int32_t* q,
+                                    const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
+  if constexpr (KF <= 8) {
+    if (packed) {
+      if (dflt) return launch_hist_kfs<K, KF, true, true>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+      return launch_hist_kfs<K, KF, false, true>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    }
+  }
+  if (dflt) return launch_hist_kfs<K, KF, true, false>(ctx, p, hc, bins, nullptr, dflt, q, rows, use_rows, s, hist, cnt);
+  return launch_hist_kfs<K, KF, false, false>(ctx, p, hc, bins, nullptr, dflt, q, rows, use_rows, s, hist, cnt);
 }
 
 template <int K>
 static gbdtmo_status launch_hist(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
-                                 const int32_t* dflt, const int32_t* q, const int32_t* rows, int use_rows, const State& s,
-                                 int64_t* hist, int32_t* cnt) {
+                                 const uint8_t* packed, const int32_t* dflt, const int32_t* q, const int32_t* rows,
+                                 int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
   switch (hc.k) {
-    case 24: return launch_hist_kf<K, 24>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 16: return launch_hist_kf<K, 16>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 12: return launch_hist_kf<K, 12>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 8: return launch_hist_kf<K, 8>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 6: return launch_hist_kf<K, 6>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 4: return launch_hist_kf<K, 4>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 3: return launch_hist_kf<K, 3>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    case 2: return launch_hist_kf<K, 2>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
-    default: return launch_hist_kf<K, 1>(ctx, p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt);
+    case 24: return launch_hist_kf<K, 24>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 16: return launch_hist_kf<K, 16>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 12: return launch_hist_kf<K, 12>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 8: return launch_hist_kf<K, 8>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 6: return launch_hist_kf<K, 6>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 4: return launch_hist_kf<K, 4>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 3: return launch_hist_kf<K, 3>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    case 2: return launch_hist_kf<K, 2>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
+    default: return launch_hist_kf<K, 1>(ctx, p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt);
   }
+}
+
+// Tile-packed copy of the bins: packed[(t * n + i) * 8 + j] = bins[i * ld + k t + j] for
+// j < k (features of tile t), 0 above.  Threads walk (row, tile) with the tile fastest, so a
+// warp reads one row's bins contiguously; the 8-byte writes of consecutive rows of a plane
+// merge in L2.  Once per dataset (like gbdtmo_bin).
+__global__ void k_pack_bins(gbdtmo_problem p, int k, int n_ft, const uint8_t* __restrict__ bins,
+                            uint64_t* __restrict__ packed) {
+  const int64_t total = p.n * (int64_t)n_ft;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += stride) {
+    const int64_t i = e / n_ft;
+    const int t = (int)(e - i * n_ft);
+    const uint8_t* src = bins + i * p.ld_bins + (int64_t)t * k;
+    const int kk = min(k, p.m - t * k);
+    uint64_t v = 0;
+    for (int j = 0; j < kk; ++j) v |= (uint64_t)__ldg(src + j) << (8 * j);
+    packed[(int64_t)t * p.n + i] = v;
+  }
+}
+
+gbdtmo_status build_hist_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t level, const uint8_t* bins,
+                              const uint8_t* packed, const int32_t* dflt, const int32_t* q, void* state,
+                              int64_t* hist, int32_t* cnt) {
+  State s = state_view(*p, state);
+  HistCfg hc = hist_config(*p);
+  const int64_t LN = int64_t(1) << level;
+  int gx = (int)(2 * ctx->num_sms / (LN > 1 ? LN / 2 : 1));
+  if (gx < 8) gx = 8;
+  GB_LAUNCH(k_zero_build, dim3(gx, (unsigned)LN), 256, 0, *p, level, s, hist, cnt);
+  const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
+  const int use_rows = level > 0;
+  gbdtmo_status st;
+  if (ctx->hist_kernel == 1 && !dflt) {
+    st = launch_hist_diag(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
+  } else if (ctx->hist_kernel == 2 && !dflt && hist_tma_supported(*p, bins)) {
+    st = launch_hist_tma(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
+  } else switch (hc.K) {
+    case 4: st = launch_hist<4>(ctx, *p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt); break;
+    case 8: st = launch_hist<8>(ctx, *p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt); break;
+    default: st = launch_hist<16>(ctx, *p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt); break;
+  }
+  if (st != GBDTMO_OK || ctx->gmem_max_rows <= 0) return st;
+  if (dflt) GB_LAUNCH(k_hist_gmem<true>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  else GB_LAUNCH(k_hist_gmem<false>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  return GBDTMO_OK;
 }
 
 }  // namespace gbdtmo
@@ -328,24 +394,38 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
   GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
   GB_CHECK_ARG(bins && q && state && hist && cnt, "null pointer");
   GB_CHECK_ARG(((uintptr_t)bins & 7) == 0, "bins must be 8-byte aligned");
-  State s = state_view(*p, state);
-  HistCfg hc = hist_config(*p);
-  const int64_t LN = int64_t(1) << level;
-  int gx = (int)(2 * ctx->num_sms / (LN > 1 ? LN / 2 : 1));
-  if (gx < 8) gx = 8;
-  GB_LAUNCH(k_zero_build, dim3(gx, (unsigned)LN), 256, 0, *p, level, s, hist, cnt);
-  const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
-  const int use_rows = level > 0;
-  gbdtmo_status st;
-  if (ctx->hist_kernel == 1 && !dflt) {
-    st = launch_hist_diag(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
-  } else switch (hc.K) {
-    case 4: st = launch_hist<4>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
-    case 8: st = launch_hist<8>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
-    default: st = launch_hist<16>(ctx, *p, hc, bins, dflt, q, rows, use_rows, s, hist, cnt); break;
-  }
-  if (st != GBDTMO_OK || ctx->gmem_max_rows <= 0) return st;
-  if (dflt) GB_LAUNCH(k_hist_gmem<true>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
-  else GB_LAUNCH(k_hist_gmem<false>, ctx->num_sms * 8, 256, 0, *p, bins, dflt, q, rows, use_rows, s, hist, cnt);
+  return build_hist_impl(ctx, p, level, bins, nullptr, dflt, q, state, hist, cnt);
+}
+
+extern "C" gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
+                                                  const uint8_t* bins, const uint8_t* packed, const int32_t* dflt,
+                                                  const int32_t* q, void* state, int64_t* hist, int32_t* cnt) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  const char* bad = check_problem(p);
+  GB_CHECK_ARG(!bad, bad ? bad : "");
+  GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
+  GB_CHECK_ARG(bins && packed && q && state && hist && cnt, "null pointer");
+  GB_CHECK_ARG(((uintptr_t)bins & 7) == 0 && ((uintptr_t)packed & 7) == 0, "bins / packed must be 8-byte aligned");
+  GB_CHECK_ARG(hist_packable(*p), "feature tiles wider than 8 features: no packed layout (gbdtmo_packed_bins_bytes = 0)");
+  return build_hist_impl(ctx, p, level, bins, packed, dflt, q, state, hist, cnt);
+}
+
+extern "C" size_t gbdtmo_packed_bins_bytes(const gbdtmo_problem* p) {
+  if (check_problem(p) || !hist_packable(*p)) return 0;
+  return (size_t)hist_config(*p).n_ft * (size_t)p->n * 8;
+}
+
+extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p, const uint8_t* bins,
+                                          uint8_t* packed) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  const char* bad = check_problem(p);
+  GB_CHECK_ARG(!bad, bad ? bad : "");
+  GB_CHECK_ARG(bins && packed, "null pointer");
+  GB_CHECK_ARG(((uintptr_t)packed & 7) == 0, "packed must be 8-byte aligned");
+  GB_CHECK_ARG(hist_packable(*p), "feature tiles wider than 8 features: no packed layout (gbdtmo_packed_bins_bytes = 0)");
+  const HistCfg hc = hist_config(*p);
+  GB_LAUNCH(k_pack_bins, ctx->num_sms * 8, 256, 0, *p, hc.k, hc.n_ft, bins, reinterpret_cast<uint64_t*>(packed));
   return GBDTMO_OK;
 }

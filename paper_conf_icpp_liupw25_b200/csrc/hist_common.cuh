@@ -33,6 +33,15 @@ __device__ __forceinline__ uint32_t byte_of(const uint64_t (&sw)[SW], int j) {  
   return __byte_perm(half, 0u, 0x4440u | (uint32_t)(j & 3));                     // PRMT: one byte, zero-extended
 }
 
+// PRMT in its default mode, where a selector nibble with bit 3 set replicates the sign bit of
+// the selected byte (__byte_perm ignores that bit): prmt_sx(x, 0x4410) = x & 0xFFFF,
+// prmt_sx(x, 0xBB32) = x >> 16 (arithmetic).
+__device__ __forceinline__ uint32_t prmt_sx(uint32_t x, uint32_t sel) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(r) : "r"(x), "r"(sel));
+  return r;
+}
+
 // Shared-memory atomic add without return (SASS ATOMS.ADD) at a 32-bit shared address.
 __device__ __forceinline__ void red_shared_add(uint32_t addr, uint32_t v) {
   asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");

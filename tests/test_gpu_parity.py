@@ -202,7 +202,8 @@ def test_grad_matches_oracle(orc, pkg, ctx, case):
 
 # ------------------------------------------------------------------------ histograms
 
-@pytest.mark.parametrize("case,hk", [(c, k) for k in (0, 1) for c in ("C1", "C3s", "C5s", "C2s", "C4s")])
+@pytest.mark.parametrize("case,hk", [(c, k) for k in (0, 1) for c in ("C1", "C3s", "C5s", "C2s", "C4s")] +
+                         [(c, 2) for c in ("C3s", "C5s", "C2s", "C4s")])
 def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
     """Every level's histograms (built and derived by subtraction) vs the oracle's direct
     per-node histograms over the oracle's node rows; exact on tree-1 dyadic MSE inputs."""
@@ -261,7 +262,9 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
     ("C1", False, 0, 2000, 0), ("C2s", False, 0, 4000, 0), ("C2s", True, 256, 2500, 0),     # sort-and-segment small nodes
     ("C3s", False, 0, 9000, 0), ("C5s", False, 0, 6000, 0),
     ("C1", False, 0, 0, 1), ("C2s", False, 0, 0, 1), ("C3s", False, 0, 0, 1), ("C4s", False, 0, 0, 1),  # diagonal
-    ("C5s", False, 0, 0, 1), ("S300s", False, 0, 0, 1), ("C2s", False, 3000, 128, 1)])
+    ("C5s", False, 0, 0, 1), ("S300s", False, 0, 0, 1), ("C2s", False, 3000, 128, 1),
+    ("C2s", False, 0, 0, 2), ("C3s", False, 0, 0, 2), ("C4s", False, 0, 0, 2), ("C5s", False, 0, 0, 2),  # TMA-staged
+    ("S300s", False, 0, 0, 2), ("C5s", False, 5000, 0, 2), ("C3s", False, 0, 9000, 2)])
 def test_trees_and_predictions_vs_oracle(orc, pkg, ctx, case, sparse, gmem, small, hk):
     w = CASES[case]
     X, Y = _inputs(w)
@@ -382,3 +385,38 @@ def test_graph_replay_equals_eager(pkg, ctx):
         b.step_graph()
     torch.cuda.synchronize()
     assert torch.equal(a.pred, b.pred)
+
+
+@pytest.mark.parametrize("case,sparse", [("C3s", False), ("C5s", False), ("C2s", True), ("C4s", False)])
+def test_packed_bins_layout_and_equivalence(orc, pkg, ctx, case, sparse):
+    """gbdtmo_pack_bins writes the documented [tile][row][8] layout (checked against a numpy
+    re-layout of the oracle's bins), and training from the packed copy gives exactly the trees and
+    predictions of the row-major path (integer histograms: bit-equal), which equal the oracle's."""
+    w = CASES[case]
+    X, Y = _inputs(w)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)          # bins [m][n]
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+    yd = torch.from_numpy(Y).to(DEV)
+    kw = dict(sparse_default=sparse, gmem_max_rows=0, small_max_rows=0, hist_kernel=0)
+    bp = pkg.Booster(ctx, ds, yd, _params(pkg, w), packed_bins=True, **kw)
+    torch.cuda.synchronize()
+    n, m, k = w.n, w.m, 6                                # K = 16 tiles of 6 features at B = 256 (hist_config)
+    nt = (m + k - 1) // k
+    assert bp.packed.numel() == nt * n * 8
+    want = np.zeros((nt, n, 8), dtype=np.uint8)
+    for f in range(m):
+        want[f // k, :, f % k] = bins[f]
+    np.testing.assert_array_equal(bp.packed.view(nt, n, 8).cpu().numpy(), want)
+    br = pkg.Booster(ctx, ds, yd, _params(pkg, w), packed_bins=False, **kw)
+    bp.fit()
+    br.fit()
+    torch.cuda.synchronize()
+    assert torch.equal(bp.pred, br.pred)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    for t in range(w.T):
+        a, b = to_np(bp.trees[t]), to_np(br.trees[t])
+        for key in ("node_state", "feature", "bin", "n_rows"):
+            np.testing.assert_array_equal(a[key], b[key])
+        assert not compare_trees(a, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t])
+    assert np.max(np.abs(bp.pred.cpu().numpy() - ref["pred"])) <= 1e-4

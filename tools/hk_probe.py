@@ -34,7 +34,10 @@ def main():
         V = w.d * (2 if w.loss == gen.LOSS_SOFTMAX else 1)
         gm = pkg.booster.variant_threshold(V, w.m, "gmem_max_rows", n=w.n)
         sm = pkg.booster.variant_threshold(V, w.m, "small_max_rows", n=w.n)
-        res = {hk: round(time_trees(ctx, ds, Y, w, gm, sm, warm=2, timed=3, hk=hk), 3) for hk in (0, 1, 0, 1)}
+        kernels = [int(k) for k in os.environ.get("HK", "0,1").split(",")]
+        res = {}
+        for hk in kernels + kernels:
+            res.setdefault(hk, []).append(round(time_trees(ctx, ds, Y, w, gm, sm, warm=2, timed=3, hk=hk), 3))
         print(json.dumps({"workload": w.name, "gmem": gm, "small": sm, "ms_per_tree_by_hist_kernel": res}), flush=True)
         del ds, Y
         torch.cuda.empty_cache()

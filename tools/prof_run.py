@@ -27,7 +27,10 @@ def main():
     del X
     Y = torch.from_numpy(gen.targets_host(w)).to(dev)
     P = pkg.Params(loss=w.loss, T=trees, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
-    b = pkg.Booster(ctx, ds, Y, P)
+    kw = {}
+    if os.environ.get("PACKED") is not None:       # A/B: PACKED=0 row-major bins, PACKED=1 tile-packed
+        kw["packed_bins"] = os.environ["PACKED"] == "1"
+    b = pkg.Booster(ctx, ds, Y, P, **kw)
     for _ in range(trees):
         b.step()
     torch.cuda.synchronize()

@@ -90,7 +90,14 @@ struct HistCfg {
   int smem;   // bytes of dynamic shared memory
 };
 
-__host__ __device__ inline int hist_cnt_words(int K, int k, int B) { return k * B; }   // counts[k][B]
+#ifndef GBDTMO_HIST_LCNT
+#define GBDTMO_HIST_LCNT 0   // (A/B) 1: K = 16 tiles count in the accumulation loop, bank-per-lane table
+#endif
+__host__ __device__ inline bool hist_lane_counts(int K, int k) { return GBDTMO_HIST_LCNT && K == 16 && k <= 8; }
+// counts[k][B] int32, or with lane counts a [ceil(B/2)][32] table of 16-bit counter pairs
+__host__ __device__ inline int hist_cnt_words(int K, int k, int B) {
+  return hist_lane_counts(K, k) ? ((B + 1) / 2) * 32 : k * B;
+}
 
 __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   HistCfg c;

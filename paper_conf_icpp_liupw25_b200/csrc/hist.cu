@@ -38,6 +38,14 @@ namespace gbdtmo {
 // shifts it, counts it (CNT) and parks the bins in the scratch; then the K groups of
 // 32/K rows are accumulated, lanes (row, channel) reading their bins back with one LDS and
 // their q value from a batch-wide prefetch.
+template <int KF>
+__device__ __forceinline__ int dfl_of(const int (&dfl)[KF], int j) {   // dfl[j], j runtime
+  int v = -1;
+#pragma unroll
+  for (int u = 0; u < KF; ++u) v = (u == j) ? dfl[u] : v;
+  return v;
+}
+
 template <int K, int KF, bool SKIP, bool PACKED>
 __global__ void __launch_bounds__(kHistThreads, 1)
 k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const uint8_t* __restrict__ packed,
@@ -54,6 +62,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #ifndef GBDTMO_HIST_SB
 #define GBDTMO_HIST_SB 8
 #endif
+#ifndef GBDTMO_HIST_SHFL
+#define GBDTMO_HIST_SHFL 0         // (A/B) 1: phase 2 takes the bins by SHFL, no scratch round trip
+#endif
   constexpr int SB = G < GBDTMO_HIST_SB ? G : GBDTMO_HIST_SB;   // groups per q-prefetch sub-batch
   constexpr int RS = KF * 2 * K;               // limb words per bin
   constexpr int NW = PACKED ? 1 : HistRow<KF>::NW, SW = PACKED ? 1 : HistRow<KF>::SW;
@@ -64,7 +75,8 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   const int tiles = hc.n_ft * hc.n_ct;
   const int nitems = s.misc[MISC_CHUNK_COUNT] * tiles;
   const int limb_words = B * RS;
-  const int cnt_words = B * KF;
+  constexpr bool LCNT = GBDTMO_HIST_LCNT && K == 16 && KF <= 8;
+  const int cnt_words = LCNT ? ((B + 1) >> 1) * 32 : B * KF;
   uint64_t* scratch = reinterpret_cast<uint64_t*>(sm + limb_words + cnt_words + ((limb_words + cnt_words) & 1)) +
                       (size_t)warp * 32 * SW;
   const int slotA = c + ((ri & 1) ? K : 0), slotB = slotA ^ K;
@@ -75,6 +87,11 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   // limb selectors for PRMT(q, sel, 0): lo = bytes 0-1 zero-extended (0x4410), hi = bytes 2-3
   // sign-extended (0xBB32); even rows add (lo, hi) at (slotA, slotB), odd rows (hi, lo)
   const uint32_t selA = (ri & 1) ? 0xBB32u : 0x4410u, selB = (ri & 1) ? 0x4410u : 0xBB32u;
+  // lane counts (LCNT): lane (ri, c < 2 KF) counts feature cj of the earlier (c < KF) or later
+  // row pair of every two, into column 16 ri + c of the [bin/2][32] table (bank = column)
+  const int cj = c < KF ? c : c - KF;
+  const uint32_t acol = sbase + 4u * (limb_words + 16 * ri + c);
+  const uint32_t cshift = 8u * cj;
 
   for (;;) {
     if (threadIdx.x == 0) sh_item = atomicAdd(&s.misc[MISC_WORK_COUNTER], 1);
@@ -149,7 +166,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
             sw[i] = keep >= 8 ? sw[i] : keep <= 0 ? 0ull : (sw[i] & ((1ull << (8 * keep)) - 1));
           }
         }
-        if (do_cnt && !GBDTMO_HIST_NOCOUNT) {
+        if (!LCNT && do_cnt && !GBDTMO_HIST_NOCOUNT) {
 #pragma unroll
           for (int j = 0; j < KF; ++j) {         // features j >= kk land in slots never flushed
             const uint32_t bin = byte_of<SW>(sw, j);
@@ -161,6 +178,8 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       for (int i = 0; i < SW; ++i) scratch[lane * SW + i] = sw[i];
       __syncwarp();
       // ---- phase 2: groups of RPI rows x K channels
+      const bool cnt_on = LCNT && do_cnt && c < 2 * KF && cj < kk;
+      uint64_t bprev = 0;
 #pragma unroll
       for (int t0 = 0; t0 < G; t0 += SB) {
         int qn[SB];
@@ -170,8 +189,24 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         for (int t = 0; t < SB; ++t) {
           const int i = (t0 + t) * RPI + ri;
           uint64_t bw[SW];
+          if (GBDTMO_HIST_SHFL && SW == 1) {       // (A/B) bins by shuffle instead of the scratch
+            const uint32_t w0 = __shfl_sync(0xffffffffu, (uint32_t)sw[0], i);
+            const uint32_t w1 = KF > 4 ? __shfl_sync(0xffffffffu, (uint32_t)(sw[0] >> 32), i) : 0u;
+            bw[0] = ((uint64_t)w1 << 32) | w0;
+          } else {
 #pragma unroll
-          for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
+            for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
+          }
+          if (LCNT) {
+            if ((t0 + t) & 1) {
+              const uint64_t w = c < KF ? bprev : bw[0];
+              const int row = c < KF ? i - 2 : i;
+              const uint32_t bin = (uint32_t)(w >> cshift) & 0xFFu;
+              if (cnt_on && b0 + row < end && (!SKIP || (int)bin != dfl_of(dfl, cj)))
+                red_shared_add(acol + (bin >> 1) * 128u, 1u << ((bin & 1) << 4));
+            }
+            bprev = bw[0];
+          }
           const uint32_t va = prmt_sx((uint32_t)qv[t], selA);
           const uint32_t vb = prmt_sx((uint32_t)qv[t], selB);
 #pragma unroll
@@ -213,7 +248,16 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {
-        const uint32_t nv = sm[limb_words + e];                    // counts[j][b], e = j * B + b
+        uint32_t nv;                                               // count of (feature j, bin b), e = j * B + b
+        if (LCNT) {
+          const int j = e / B, b = e - j * B;
+          const uint32_t* cw = sm + limb_words + (b >> 1) * 32;
+          const int sh = 16 * (b & 1);
+          nv = ((cw[j] >> sh) & 0xFFFFu) + ((cw[j + KF] >> sh) & 0xFFFFu) + ((cw[16 + j] >> sh) & 0xFFFFu) +
+               ((cw[16 + j + KF] >> sh) & 0xFFFFu);
+        } else {
+          nv = sm[limb_words + e];                                 // counts[j][b]
+        }
         if (sole) cnt[gbase + e] = (int32_t)nv;
         else if (nv) atomicAdd(&cnt[gbase + e], (int32_t)nv);
       }

@@ -234,6 +234,43 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int64_t slot = ch.x;
     const bool sole = ch.w != 0;
     const int64_t gbase = (slot * m + f0) * (int64_t)B;        // (slot, f0, bin 0)
+    if (K == 16) {
+      // Warp-transposed flush: the limb records are bin-major with bank = slot, the global
+      // histogram is bin-minor.  A warp takes (feature j, 32 bins): reads them with lanes = slots
+      // (conflict-free), writes each bin's 32 slots back XOR-swizzled by the bin, reads them again
+      // with lanes = bins (conflict-free), and stores 32 consecutive bins per channel (2 lines per
+      // instruction instead of 32).
+      const int nblk = (B + 31) >> 5;
+      for (int task = warp; task < kk * nblk; task += nwarps) {
+        const int j = task / nblk, bb = (task - j * nblk) << 5;
+        uint32_t* rec = sm + j * 2 * K;                        // + b * RS + slot
+#pragma unroll
+        for (int h = 0; h < 32; h += 16) {
+          uint32_t v[16];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) v[u] = (bb + h + u < B) ? rec[(bb + h + u) * RS + lane] : 0u;
+          __syncwarp();
+#pragma unroll
+          for (int u = 0; u < 16; ++u)
+            if (bb + h + u < B) rec[(bb + h + u) * RS + (lane ^ (h + u))] = v[u];
+        }
+        __syncwarp();
+        const int b = bb + lane;
+        if (b < B) {
+          const uint32_t* rb = rec + b * RS;
+          int64_t* dst = &hist[((slot * m + f0 + j) * V + c0) * (int64_t)B + b];
+#pragma unroll 4
+          for (int cc = 0; cc < K; ++cc) {
+            if (c0 + cc >= V) break;
+            const uint32_t los = rb[cc ^ lane], his = rb[(K + cc) ^ lane];
+            const long long v = (long long)(int32_t)his * 65536LL + (long long)los;
+            if (sole) dst[(int64_t)cc * B] = v;
+            else if (v != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + (int64_t)cc * B), (unsigned long long)v);
+          }
+        }
+        __syncwarp();
+      }
+    } else {
     const int total = kk * B * K;
     for (int e = threadIdx.x; e < total; e += blockDim.x) {
       const int cc = e % K, jb = e / K;                        // jb = j * B + b
@@ -245,6 +282,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
       int64_t* dst = &hist[((slot * m + f0 + j) * V + c0 + cc) * B + b];   // channel-major [f][c][b]
       if (sole) *dst = v;
       else if (v != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst), (unsigned long long)v);
+    }
     }
     if (do_cnt) {
       for (int e = threadIdx.x; e < kk * B; e += blockDim.x) {

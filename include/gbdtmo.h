@@ -208,9 +208,11 @@ gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t
  * features (k from the problem's shape, at most 8 for a packed layout); with the row-major
  * matrix every row of a tile is its own cache line, so a warp's 32 gathered rows cost 32-64 L1
  * wavefronts per load.  The packed copy stores each tile's bins contiguously per row:
- *   packed uint8 [n_tiles][n][8]:  packed[(t * n + i) * 8 + j] = bins[i * ld + k t + j] (j < k),
- *                                  0 for j >= k or k t + j >= m,
- * so adjacent rows are adjacent 8-byte words.  gbdtmo_packed_bins_bytes: bytes of `packed`, 0 when
+ *   packed uint8 [ceil(n_tiles/4)][n][4][8]:
+ *     packed[(((t / 4) * n + i) * 4 + t % 4) * 8 + j] = bins[i * ld + k t + j]  (j < k),
+ *     0 for j >= k or k t + j >= m,
+ * so one row's bins for 4 consecutive tiles are one 32-byte sector and adjacent rows are adjacent
+ * sectors.  gbdtmo_packed_bins_bytes: bytes of `packed`, 0 when
  * the problem's tiles are wider than 8 features (then use gbdtmo_build_hist).  The caller owns
  * `packed`; gbdtmo_pack_bins fills it from `bins` (once per dataset and problem shape).
  * gbdtmo_build_hist_packed = gbdtmo_build_hist reading the tile bins from `packed` (and `bins`

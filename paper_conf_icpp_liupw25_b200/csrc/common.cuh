@@ -120,8 +120,15 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   return c;
 }
 
-// Tile-packed bins (gbdtmo_pack_bins): uint8 [n_ft][n][8], slot (t, i) = bins of features
-// [k t, k t + k) of row i, zero padded; only for tiles of <= 8 features.
+// Tile-packed bins (gbdtmo_pack_bins): uint8 [ceil(n_ft/G)][n][G][8], G = kPackGroup tiles per
+// row group; word (t, i) = bins of features [k t, k t + k) of row i, zero padded; only for tiles
+// of <= 8 features.  G = 4: a 32-byte sector holds one row's bins for 4 consecutive tiles, which
+// the work order runs concurrently, so gathered rows at deep levels fetch each sector once (with
+// G = 1 every (row, tile) was its own sector: 79 GB of DRAM reads in one C5 level-7 launch).
+#ifndef GBDTMO_PACK_GROUP
+#define GBDTMO_PACK_GROUP 4
+#endif
+constexpr int kPackGroup = GBDTMO_PACK_GROUP;
 __host__ __device__ inline bool hist_packable(const gbdtmo_problem& p) { return hist_config(p).k <= 8; }
 
 // ------------------------------------------------------------- state layout

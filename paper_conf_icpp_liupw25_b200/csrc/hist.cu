@@ -117,8 +117,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 
     const int beg = ch.y, end = ch.z;
     const int o = PACKED ? 0 : f0 & 7;
-    const uint8_t* bbase = PACKED ? packed + (int64_t)ft * p.n * 8 : bins + (f0 & ~7);
-    const int64_t rstride = PACKED ? 8 : ld;
+    const uint8_t* bbase = PACKED ? packed + ((int64_t)(ft / kPackGroup) * p.n * kPackGroup + ft % kPackGroup) * 8
+                                  : bins + (f0 & ~7);
+    const int64_t rstride = PACKED ? 8 * kPackGroup : ld;
     const bool chan_on = (c0 + c) < V;
     const int32_t* qc = q + c0 + c;
     // cross-batch pipeline: row ids two batches ahead, bin windows one batch ahead, q one
@@ -416,22 +417,23 @@ static gbdtmo_status launch_hist(Ctx* ctx, const gbdtmo_problem& p, const HistCf
   }
 }
 
-// Tile-packed copy of the bins: packed[(t * n + i) * 8 + j] = bins[i * ld + k t + j] for
-// j < k (features of tile t), 0 above.  Threads walk (row, tile) with the tile fastest, so a
-// warp reads one row's bins contiguously; the 8-byte writes of consecutive rows of a plane
-// merge in L2.  Once per dataset (like gbdtmo_bin).
+// Tile-packed copy of the bins, groups of kPackGroup tiles per row:
+//   packed[((t / G) * n + i) * G + t % G] (8-byte words) = bins of features [k t, k t + k) of row i
+// Threads walk (row, tile) with the tile fastest: a warp reads one row's bins contiguously and
+// writes its 32-byte groups contiguously.  Once per dataset (like gbdtmo_bin).
 __global__ void k_pack_bins(gbdtmo_problem p, int k, int n_ft, const uint8_t* __restrict__ bins,
                             uint64_t* __restrict__ packed) {
-  const int64_t total = p.n * (int64_t)n_ft;
+  const int n_g = (n_ft + kPackGroup - 1) / kPackGroup;
+  const int64_t total = p.n * (int64_t)n_g * kPackGroup;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += stride) {
-    const int64_t i = e / n_ft;
-    const int t = (int)(e - i * n_ft);
+    const int64_t i = e / (n_g * kPackGroup);
+    const int t = (int)(e - i * n_g * kPackGroup);
     const uint8_t* src = bins + i * p.ld_bins + (int64_t)t * k;
     const int kk = min(k, p.m - t * k);
     uint64_t v = 0;
     for (int j = 0; j < kk; ++j) v |= (uint64_t)__ldg(src + j) << (8 * j);
-    packed[(int64_t)t * p.n + i] = v;
+    packed[((int64_t)(t / kPackGroup) * p.n + i) * kPackGroup + t % kPackGroup] = v;
   }
 }
 
@@ -495,7 +497,8 @@ extern "C" gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx c, const gbdtmo_pro
 
 extern "C" size_t gbdtmo_packed_bins_bytes(const gbdtmo_problem* p) {
   if (check_problem(p) || !hist_packable(*p)) return 0;
-  return (size_t)hist_config(*p).n_ft * (size_t)p->n * 8;
+  const size_t groups = (size_t)(hist_config(*p).n_ft + kPackGroup - 1) / kPackGroup;
+  return groups * (size_t)p->n * 8 * kPackGroup;
 }
 
 extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p, const uint8_t* bins,

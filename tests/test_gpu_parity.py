@@ -402,11 +402,13 @@ def test_packed_bins_layout_and_equivalence(orc, pkg, ctx, case, sparse):
     torch.cuda.synchronize()
     n, m, k = w.n, w.m, 6                                # K = 16 tiles of 6 features at B = 256 (hist_config)
     nt = (m + k - 1) // k
-    assert bp.packed.numel() == nt * n * 8
-    want = np.zeros((nt, n, 8), dtype=np.uint8)
+    ng = (nt + 3) // 4                                   # groups of 4 tiles per row
+    assert bp.packed.numel() == ng * n * 4 * 8
+    want = np.zeros((ng, n, 4, 8), dtype=np.uint8)
     for f in range(m):
-        want[f // k, :, f % k] = bins[f]
-    np.testing.assert_array_equal(bp.packed.view(nt, n, 8).cpu().numpy(), want)
+        t = f // k
+        want[t // 4, :, t % 4, f % k] = bins[f]
+    np.testing.assert_array_equal(bp.packed.view(ng, n, 4, 8).cpu().numpy(), want)
     br = pkg.Booster(ctx, ds, yd, _params(pkg, w), packed_bins=False, **kw)
     bp.fit()
     br.fit()

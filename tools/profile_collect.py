@@ -69,34 +69,32 @@ def main():
         subprocess.run(["cp", lc, os.path.join(PROF, f"{tag}_launches_bench_c5.csv")])
         launch_summary(lc, os.path.join(PROF, f"{tag}_launches_bench_c5_summary.txt"))
     for name in ("hist", "fs"):
-        rep = os.path.join(OUT, f"{tag}_prof_{name}_c5.ncu-rep")
-        if os.path.exists(rep):
-            txt = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_summary.py"), rep, "--sass", "30"],
-                                 capture_output=True, text=True).stdout
-            open(os.path.join(PROF, f"{tag}_ncu_{name}_c5.txt"), "w").write(txt)
-            if name == "hist":
-                # dram bytes per launch (average over the captured launches) for bench.py's roofline.traffic
-                raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-                rr = list(csv.reader(raw.splitlines()))
-                h, units = rr[0], rr[1]
-                tot, cnt = 0.0, 0
-                for r in rr[2:]:
-                    try:
-                        rd = float(r[h.index("dram__bytes_read.sum")].replace(",", ""))
-                        wr = float(r[h.index("dram__bytes_write.sum")].replace(",", ""))
-                    except (ValueError, IndexError):
-                        continue
-                    if rd != rd or wr != wr:      # NaN: a replay that failed to collect
-                        continue
-                    unit = units[h.index("dram__bytes_read.sum")]
-                    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
-                    tot += (rd + wr) * scale
-                    cnt += 1
-                if cnt:
-                    json.dump({"workload": "C5-high-dim-feature-partitioned", "kernel": "k_hist_smem",
-                               "dram_bytes_per_launch": tot / cnt, "launches": cnt,
-                               "source": f"profiles/{tag}_ncu_hist_c5.txt (ncu --set full, one tree)"},
-                              open(os.path.join(PROF, "hist_traffic.json"), "w"), indent=1)
+        txt = os.path.join(OUT, f"{tag}_ncu_{name}_c5.txt")
+        if os.path.exists(txt):
+            subprocess.run(["cp", txt, os.path.join(PROF, f"{tag}_ncu_{name}_c5.txt")])
+        rawp = os.path.join(OUT, f"{tag}_prof_{name}_c5_raw.csv")
+        if name == "hist" and os.path.exists(rawp):
+            # dram bytes per launch (average over the captured launches) for bench.py's roofline.traffic
+            rr = list(csv.reader(open(rawp)))
+            h, units = rr[0], rr[1]
+            tot, cnt = 0.0, 0
+            for r in rr[2:]:
+                try:
+                    rd = float(r[h.index("dram__bytes_read.sum")].replace(",", ""))
+                    wr = float(r[h.index("dram__bytes_write.sum")].replace(",", ""))
+                except (ValueError, IndexError):
+                    continue
+                if rd != rd or wr != wr:      # NaN: a replay that failed to collect
+                    continue
+                unit = units[h.index("dram__bytes_read.sum")]
+                scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+                tot += (rd + wr) * scale
+                cnt += 1
+            if cnt:
+                json.dump({"workload": "C5-high-dim-feature-partitioned", "kernel": "k_hist_smem",
+                           "dram_bytes_per_launch": tot / cnt, "launches": cnt,
+                           "source": f"profiles/{tag}_ncu_hist_c5.txt (ncu --set full, one tree)"},
+                          open(os.path.join(PROF, "hist_traffic.json"), "w"), indent=1)
     bp = os.path.join(OUT, f"{tag}_bin_probe_c5.log")
     if os.path.exists(bp):
         j = last_json(bp)

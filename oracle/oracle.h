@@ -27,7 +27,8 @@
  *   oracle_leaf_value     pinned  (MSE λ=0 → sklearn leaf means)
  *   oracle_update_pred    pinned  (sklearn boosting on residuals)
  *   oracle_train (MSE)    pinned  (sklearn residual-tree boosting, λ=0)
- *   oracle_train (softmax) parity unpinned as a whole model (per-step pins only)
+ *   oracle_train (softmax) pinned  (d = 2: sklearn HistGradientBoostingClassifier, binary log loss;
+ *                                   d > 2: per-step pins only)
  */
 #ifndef GBDTMO_ORACLE_H
 #define GBDTMO_ORACLE_H

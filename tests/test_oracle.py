@@ -315,8 +315,48 @@ def test_mse_model_equals_sklearn_residual_trees(orc, D, T):
     assert np.max(np.abs(res["pred"] - pred)) < 1e-9
 
 
+@pytest.mark.parametrize("T,D,lam,lr", [(5, 4, 1.0, 0.5), (4, 3, 0.5, 0.7), (3, 5, 2.5, 0.3)])
+def test_softmax_two_class_model_equals_sklearn_hgb(orc, T, D, lam, lr):
+    """Whole softmax model pinned through its 2-class special case.  With d = 2, softmax CE with
+    the diagonal Hessian (R12, R13) gives g_1 = -g_0 = p_1 - y_1 and h_0 = h_1 = p_1 (1 - p_1),
+    p_1 = sigmoid(z_1 - z_0); Eq. (3) summed over k is then 2 G^2 / (H + lambda), so every split
+    is the binary-logistic split, and the margin z_1 - z_0 moves by 2 x (-lr G / (H + lambda))
+    per leaf.  That is scikit-learn's HistGradientBoostingClassifier (binary log
+    loss, same g/h) at learning_rate 2 lr, l2 = lambda, max_depth D, min_samples_leaf 20,
+    unlimited leaves (level-wise = leaf-wise here, R6), baseline log-odds 0 (balanced labels,
+    R10), fitted on the bin matrix (R14: integer bins bin to themselves).  sklearn keeps g/h
+    in float32, hence the 1e-6 tolerance; lambda stays >= 0.5 because with lambda -> 0 pure
+    nodes drive p to 0/1, where sklearn's float32 hessians underflow and its fixed
+    min_hessian_to_split = 1e-3 (not a model parameter of the paper) starts to bind."""
+    from sklearn.ensemble import HistGradientBoostingClassifier
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    n = X.shape[0]
+    score = np.tanh(1.3 * X[:, 0] - X[:, 3]) + 0.5 * X[:, 5] * X[:, 2] + 0.3 * X[:, 7]
+    lab = np.zeros(n, np.int64)
+    lab[np.argsort(score, kind="stable")[n // 2:]] = 1          # exactly n/2 positives
+    Y = np.stack([1.0 - lab, lab.astype(np.float64)], 1)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    assert all(len(np.unique(bins[f])) == nbins[f] for f in range(w.m))   # every bin present
+    res = orc.train(bins, nbins, w.B, Y, loss=1, T=T, D=D, lam=lam, gamma=0.0, lr=lr, min_node=20)
+    Xb = bins.T.astype(np.float64)
+    clf = HistGradientBoostingClassifier(learning_rate=2 * lr, max_iter=T, max_leaf_nodes=None, max_depth=D,
+                                         min_samples_leaf=20, l2_regularization=lam, early_stopping=False,
+                                         max_bins=255).fit(Xb, lab)
+    raw = clf._raw_predict(Xb)[:, 0]
+    margin = res["pred"][:, 1] - res["pred"][:, 0]
+    assert np.max(np.abs(raw - margin)) < 1e-6 * max(1.0, np.max(np.abs(margin)))
+    np.testing.assert_allclose(res["pred"][:, 0], -res["pred"][:, 1], rtol=0, atol=1e-12)
+    for t in range(T):
+        nodes = clf._predictors[t][0].nodes
+        assert int(res["feat"][t][0]) == int(nodes[0]["feature_idx"])
+        assert int(res["bin"][t][0]) == int(nodes[0]["bin_threshold"])
+        assert int((res["state"][t] == 2).sum()) == int(nodes["is_leaf"].sum())
+
+
 def test_train_softmax_invariants(orc):
-    # softmax model (parity unpinned as a whole): structural invariants only
+    # softmax model, d > 2: structural invariants (the model as a whole is pinned at d = 2 above;
+    # the per-step pins cover general d)
     w = gen.WORKLOADS["C2"].scaled(n=3000, m=20, T=3, D=3)
     X = gen.features_host(w, 0, w.n, 0, w.m)
     y = gen.targets_host(w, X).astype(np.float64)

@@ -50,6 +50,10 @@ def parse():
     ap.add_argument("--graph", action="store_true", help="replay each tree as a CUDA graph (1 GPU)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N > 1 (gloo: lets N ranks share one GPU for testing)")
+    ap.add_argument("--exchange", default="auto", choices=["auto", "peer", "collective"],
+                    help="N > 1 split exchange: peer = fused peer-memory exchange inside the kernels (NEXT-4), "
+                         "collective = torch.distributed all-reduces; auto = peer, verified after the warm-up "
+                         "(identical trees on every rank, no timeout) else collective")
     return ap.parse_args()
 
 
@@ -248,12 +252,31 @@ def main():
     del ds2
     del X
     torch.cuda.empty_cache()
-    booster = pkg.Booster(ctx, ds, Y, params, group=group)
+    exchange = a.exchange if a.exchange != "auto" else ("peer" if world > 1 else "collective")
+    exchange_note = None
+    try:
+        booster = pkg.Booster(ctx, ds, Y, params, group=group, exchange=exchange)
+    except Exception as ex:            # e.g. CUDA IPC unavailable: the collective path
+        if a.exchange == "peer":
+            raise
+        exchange, exchange_note = "collective", f"peer setup failed: {type(ex).__name__}: {ex}"[:200]
+        booster = pkg.Booster(ctx, ds, Y, params, group=group, exchange=exchange)
     setup_s = time.perf_counter() - t_setup
 
     # ---- warm-up
     for _ in range(a.warmup):
         booster.step()
+    if world > 1 and booster.exchange == "peer":
+        ok = peer_consistent(booster, group, dev)
+        if not ok and a.exchange == "auto":
+            exchange, exchange_note = "collective", "peer exchange failed its post-warm-up check"
+            pred0 = torch.zeros_like(booster.pred)
+            del booster
+            booster = pkg.Booster(ctx, ds, Y, params, group=group, exchange=exchange, pred=pred0)
+            for _ in range(a.warmup):
+                booster.step()
+        elif not ok:
+            raise RuntimeError("peer exchange failed its post-warm-up check")
     if a.graph and world == 1:
         booster.capture()
     torch.cuda.synchronize()
@@ -330,6 +353,7 @@ def main():
         "data": "synthetic (seeded counter-based generator, gen/); inputs in HBM, 8.2 GB bins >> 126 MB L2 (no flush needed)",
         "config": {"workload": w.name, "n": w.n, "m": w.m, "d": w.d, "B": w.B, "D": w.D,
                    "loss": "mse" if w.loss == 0 else "softmax", "parallelism": f"feature-partition x{world}",
+                   "exchange": (exchange if world > 1 else "none") + (f" ({exchange_note})" if exchange_note else ""),
                    "l2": "inputs larger than L2", "graph": bool(a.graph and world == 1)},
         "hist_share": hist_total_ms / a.steps / ms_per_tree if ms_per_tree else None,
         "hist_rows_outputs_per_s_built": rows_built * w.d / (hist_total_ms * 1e-3) if hist_ms else None,
@@ -352,7 +376,7 @@ def main():
     if not a.no_e2e:
         Yhost = Y.cpu().pin_memory()
         del Y
-        out["e2e"] = e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yhost)
+        out["e2e"] = e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yhost, exchange)
 
     if group is not None:
         dist.barrier()
@@ -368,7 +392,28 @@ def main():
     return 0
 
 
-def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh):
+def peer_consistent(booster, group, dev):
+    """After the warm-up trees: the peer window reports no expired wait on any rank, and every rank
+    holds the same trees (node states, features, bins: replicated state, so any divergence of the
+    exchange shows here)."""
+    import torch
+    import torch.distributed as dist
+    torch.cuda.synchronize()
+    _, err = booster.peer_status()
+    sig = torch.zeros(1, dtype=torch.float64, device=dev)
+    for tr in booster.trees:
+        for k in ("node_state", "feature", "bin", "n_left"):
+            v = tr[k].to(torch.float64)
+            sig += (v * torch.arange(1, v.numel() + 1, dtype=torch.float64, device=dev)).sum()
+    lo, hi = sig.clone(), sig.clone()
+    dist.all_reduce(lo, op=dist.ReduceOp.MIN, group=group)
+    dist.all_reduce(hi, op=dist.ReduceOp.MAX, group=group)
+    bad = torch.tensor([1.0 if err else 0.0], dtype=torch.float64, device=dev)
+    dist.all_reduce(bad, op=dist.ReduceOp.MAX, group=group)
+    return bool(lo.item() == hi.item()) and bad.item() == 0.0
+
+
+def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh, exchange="collective"):
     """train(): pinned host X shard + y -> H2D -> gbdtmo_bin -> K trees -> D2H of yhat and the trees."""
     import torch
     import torch.distributed as dist
@@ -386,7 +431,8 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh):
         dist.barrier()
     e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
     e0.record()
-    b = pkg.train(Xh, Yh, params, device=str(dev), ctx=ctx, group=group, f_begin=f0, m_global=w.m)
+    b = pkg.train(Xh, Yh, params, device=str(dev), ctx=ctx, group=group, f_begin=f0, m_global=w.m,
+                  exchange=exchange)
     pred_h = torch.empty(b.pred.shape, dtype=b.pred.dtype, pin_memory=True)
     pred_h.copy_(b.pred, non_blocking=True)
     model_bytes = 0

@@ -13,7 +13,7 @@
  *     for level = 0 .. D-1:
  *         gbdtmo_build_hist      (level)            (histograms of the nodes marked "build")
  *         gbdtmo_find_split      (level)            (sibling by subtraction + Eq. (3) + argmax)
- *         [N > 1: all-reduce MAX of `keys`]
+ *         [N > 1: all-reduce MAX of `keys`, or fused: gbdtmo_split_record_peer below]
  *         gbdtmo_split_record    (level)            (owner: left sums + row-direction bitmap)
  *         [N > 1: all-reduce SUM of `xchg`]
  *         gbdtmo_partition       (level)            (decisions, stable partition, next level plan)
@@ -112,7 +112,8 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *     §7); 2: row-pair tiles whose bin windows are staged in shared memory by TMA gather4
  *     (measured slower, kept as the recorded alternative).  Same results; chosen per workload
  *     shape by measurement.  1 and 2 are not used with default bins. */
-enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3 };
+enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3,
+       GBDTMO_OPT_PEER_TIMEOUT_MS = 4 /* bound of every peer-flag wait (gbdtmo_peer_*), default 30000 */ };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Number of kernels this context has launched so far (for launch accounting). */
 int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
@@ -328,6 +329,60 @@ gbdtmo_status gbdtmo_predict(gbdtmo_ctx ctx, const float* X, int64_t n, int64_t 
  * each.  Any output pointer may be NULL. */
 gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx ctx, const gbdtmo_problem* p, const void* state, int32_t level,
                                  int32_t* rows, int32_t* node_of_row, int32_t* node_begin, int32_t* node_end);
+
+/* ------------------------------------- (e) / NEXT-4: fused peer-memory exchange (multi-GPU)
+ *
+ * The feature-partitioned scheme (each GPU owns a feature shard, finds its best
+ * split, the global best is agreed across GPUs) without host-issued collectives.  Every rank
+ * owns one "window" of device memory, allocated by the library and mapped by all ranks through
+ * CUDA IPC (NVLink / NVSwitch peer loads on a multi-GPU box).  Per level:
+ *   gbdtmo_find_split / gbdtmo_search_small   with keys = this level's window keys
+ *                                              (gbdtmo_peer_buffers): written in place;
+ *   gbdtmo_split_record_peer                   its kernel publishes a flag, waits for every
+ *                                              peer's, and takes each node's key as the max over
+ *                                              the N windows (= MAX all-reduce), then writes the
+ *                                              owner's records + bitmap into the own window;
+ *   gbdtmo_partition_peer                      its first kernel publishes / waits likewise and
+ *                                              sums the N windows' records + bitmaps (= SUM
+ *                                              all-reduce) into xchg_merged, then partitions.
+ * Results are identical to the all-reduce path (same keys, same sums).  Flags are epoch counters
+ * kept in device memory, so trees captured in CUDA graphs replay correctly.  Waits are bounded
+ * (GBDTMO_OPT_PEER_TIMEOUT_MS); an expired wait records an error and the kernel continues (its
+ * outputs are then invalid) — check gbdtmo_peer_status after a run.  Windows are per level:
+ * peer_window_bytes = 512 + 8 D 2^(D-1) + 8 D xchg_count (rounded).
+ *
+ * gbdtmo_peer_open: allocates and zeroes this rank's window for problems of p's shape (n, D,
+ *   channels), returns its IPC handle (host, GBDTMO_PEER_HANDLE_BYTES bytes).  Collective in
+ *   the sense that every rank must open before any rank connects.  1 <= world <= 8.
+ * gbdtmo_peer_connect: handles = the world handles in rank order (host, world * 64 bytes;
+ *   the caller exchanges them, e.g. with torch.distributed all_gather); maps the peers' windows.
+ * gbdtmo_peer_buffers: this rank's keys [2^(D-1)] / xchg [xchg_count] of `level` in its window
+ *   (host out: device pointers, owned by the context; either pointer may be NULL).
+ * gbdtmo_peer_status: synchronous read of the window's epoch (exchanges completed) and error
+ *   word (0 = none; else (epoch << 8) | phase, phase 1 = keys, 2 = records).
+ * gbdtmo_peer_close: unmaps and frees (also done by gbdtmo_destroy).  Synchronises the device. */
+#define GBDTMO_PEER_HANDLE_BYTES 64
+size_t        gbdtmo_peer_window_bytes(const gbdtmo_problem* p);
+gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t rank, int32_t world,
+                               uint8_t* handle /* host out, 64 bytes */);
+gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx ctx, const uint8_t* handles /* host, world * 64 bytes */);
+gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                  uint64_t** keys /* host out */, int64_t** xchg /* host out */);
+gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx ctx, int64_t* epoch /* host */, int64_t* error /* host */);
+gbdtmo_status gbdtmo_peer_close(gbdtmo_ctx ctx);
+/* gbdtmo_split_record with the key exchange fused in: keys are read from every window (no
+ * `keys` argument), records and bitmap go to the own window (no `xchg` argument); keys_merged
+ * uint64 [2^level] (out) receives the agreed keys. */
+gbdtmo_status gbdtmo_split_record_peer(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
+                                       const uint8_t* bins, const int32_t* dflt, const int32_t* q,
+                                       const float* scales, void* state,
+                                       const int64_t* hist, const int32_t* cnt,
+                                       const int64_t* parent_hist, const int32_t* parent_cnt,
+                                       uint64_t* keys_merged);
+/* gbdtmo_partition with the record exchange fused in: xchg_merged int64 [xchg_count] (out)
+ * receives the sum over the windows, then the level is partitioned from it. */
+gbdtmo_status gbdtmo_partition_peer(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level, void* state,
+                                    int64_t* xchg_merged);
 
 #ifdef __cplusplus
 }

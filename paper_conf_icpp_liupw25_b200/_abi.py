@@ -26,9 +26,12 @@ SYMBOLS = (
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
-    "gbdtmo_build_hist_packed",
+    "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
+    "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
+    "gbdtmo_partition_peer",
 )
-OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL = 1, 2, 3
+OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS = 1, 2, 3, 4
+PEER_HANDLE_BYTES = 64
 
 
 class GbdtmoError(RuntimeError):
@@ -88,6 +91,14 @@ def lib():
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_predict": ([P, P, i64, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
             "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
+            "gbdtmo_peer_window_bytes": ([PP], sz),
+            "gbdtmo_peer_open": ([P, PP, i32, i32, P], C.c_int),
+            "gbdtmo_peer_connect": ([P, P], C.c_int),
+            "gbdtmo_peer_buffers": ([P, PP, i32, C.POINTER(P), C.POINTER(P)], C.c_int),
+            "gbdtmo_peer_status": ([P, C.POINTER(i64), C.POINTER(i64)], C.c_int),
+            "gbdtmo_peer_close": ([P], C.c_int),
+            "gbdtmo_split_record_peer": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_partition_peer": ([P, PP, i32, P, P], C.c_int),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -246,3 +257,42 @@ class Context:
     def gbdtmo_rows_export(self, p, state, level, rows=None, node_of_row=None, node_begin=None, node_end=None):
         self._check(lib().gbdtmo_rows_export(self._h, C.byref(p), _ptr(state), level, _ptr(rows), _ptr(node_of_row),
                                              _ptr(node_begin), _ptr(node_end)), "gbdtmo_rows_export")
+
+    # NEXT-4: fused peer-memory exchange ------------------------------------------
+    @staticmethod
+    def gbdtmo_peer_window_bytes(p) -> int:
+        return int(lib().gbdtmo_peer_window_bytes(C.byref(p)))
+
+    def gbdtmo_peer_open(self, p, rank: int, world: int) -> bytes:
+        h = (C.c_uint8 * PEER_HANDLE_BYTES)()
+        self._check(lib().gbdtmo_peer_open(self._h, C.byref(p), rank, world, h), "gbdtmo_peer_open")
+        return bytes(h)
+
+    def gbdtmo_peer_connect(self, handles: bytes):
+        buf = (C.c_uint8 * len(handles)).from_buffer_copy(handles)
+        self._check(lib().gbdtmo_peer_connect(self._h, buf), "gbdtmo_peer_connect")
+
+    def gbdtmo_peer_buffers(self, p, level: int):
+        k, x = C.c_void_p(), C.c_void_p()
+        self._check(lib().gbdtmo_peer_buffers(self._h, C.byref(p), level, C.byref(k), C.byref(x)),
+                    "gbdtmo_peer_buffers")
+        return int(k.value), int(x.value)
+
+    def gbdtmo_peer_status(self):
+        e, r = C.c_int64(), C.c_int64()
+        self._check(lib().gbdtmo_peer_status(self._h, C.byref(e), C.byref(r)), "gbdtmo_peer_status")
+        return int(e.value), int(r.value)
+
+    def gbdtmo_peer_close(self):
+        self._check(lib().gbdtmo_peer_close(self._h), "gbdtmo_peer_close")
+
+    def gbdtmo_split_record_peer(self, p, level, bins, dflt, q, scales, state, hist, cnt, parent_hist, parent_cnt,
+                                 keys_merged):
+        self._check(lib().gbdtmo_split_record_peer(self._h, C.byref(p), level, _ptr(bins), _ptr(dflt), _ptr(q),
+                                                   _ptr(scales), _ptr(state), _ptr(hist), _ptr(cnt),
+                                                   _ptr(parent_hist), _ptr(parent_cnt), _ptr(keys_merged)),
+                    "gbdtmo_split_record_peer")
+
+    def gbdtmo_partition_peer(self, p, level, state, xchg_merged):
+        self._check(lib().gbdtmo_partition_peer(self._h, C.byref(p), level, _ptr(state), _ptr(xchg_merged)),
+                    "gbdtmo_partition_peer")

@@ -137,8 +137,13 @@ class Booster:
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
                  small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
-                 packed_bins: Optional[bool] = None):
+                 packed_bins: Optional[bool] = None, exchange: str = "collective"):
+        """exchange (only with `group`): "collective" = torch.distributed all-reduces per level;
+        "peer" = the fused peer-memory exchange (NEXT-4, gbdtmo_*_peer): the keys / records are
+        read from the other ranks' windows inside split_record / partition, no host collective."""
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
+        assert exchange in ("collective", "peer")
+        self.exchange = exchange if group is not None else "collective"
         # histogram variant selection (DESIGN.md "Variant selection"): nodes with <= gmem_max_rows
         # rows use the global-atomic variant; None = the measured table for this channel count
         V = y.shape[1] * (2 if params.loss == LOSS_SOFTMAX else 1)
@@ -188,6 +193,9 @@ class Booster:
             ctx.gbdtmo_pack_bins(self.p, ds.bins, self.packed)
         self.keys = torch.zeros(1 << max(D - 1, 0), dtype=torch.int64, device=dev)
         self.xchg = torch.zeros(ctx.gbdtmo_xchg_count(self.p), dtype=torch.int64, device=dev)
+        self.peer_keys = None
+        if self.exchange == "peer":
+            self._peer_connect()
         NH = (1 << (D + 1)) - 1
         self.NH = NH
         self.leaf = torch.empty((NH, d), dtype=torch.float64, device=dev)
@@ -195,6 +203,22 @@ class Booster:
         self.trees = []            # per tree: dict of device tensors (heap-indexed tree record)
         self._graph = None
         self.hist_events = []      # optional per-level (start, end) CUDA events around build_hist
+
+    def _peer_connect(self):
+        """Open this rank's window, exchange the IPC handles over the process group (plumbing),
+        map the peers' windows; keys of level l are then written straight into the window."""
+        import torch.distributed as dist
+        rank, world = dist.get_rank(self.group), dist.get_world_size(self.group)
+        torch.cuda.synchronize(self.device)
+        h = self.ctx.gbdtmo_peer_open(self.p, rank, world)
+        handles = [None] * world
+        dist.all_gather_object(handles, h, group=self.group)
+        self.ctx.gbdtmo_peer_connect(b"".join(handles))
+        self.peer_keys = [self.ctx.gbdtmo_peer_buffers(self.p, lvl)[0] for lvl in range(self.params.D)]
+
+    def peer_status(self):
+        """(exchanges completed, error word) of the peer window (synchronous); error 0 = healthy."""
+        return self.ctx.gbdtmo_peer_status()
 
     # ------------------------------------------------------------------ one tree
     def _level(self, lvl: int, time_hist: bool = False):
@@ -213,10 +237,17 @@ class Booster:
         if time_hist:
             e1.record()
             self.hist_events.append((e0, e1))
+        peer = self.exchange == "peer"
+        keys = self.peer_keys[lvl] if peer else self.keys     # peer: this level's window keys
         ctx.gbdtmo_find_split(p, lvl, self.ds.nbins, self.dflt, self.scales, self.state, self.hist[cur], self.cnt[cur],
-                              ph, pc, self.keys)
+                              ph, pc, keys)
         if self.small_max_rows > 0:
-            ctx.gbdtmo_search_small(p, lvl, self.ds.bins, self.q, self.ds.nbins, self.scales, self.state, self.keys)
+            ctx.gbdtmo_search_small(p, lvl, self.ds.bins, self.q, self.ds.nbins, self.scales, self.state, keys)
+        if peer:
+            ctx.gbdtmo_split_record_peer(p, lvl, self.ds.bins, self.dflt, self.q, self.scales, self.state,
+                                         self.hist[cur], self.cnt[cur], ph, pc, self.keys)
+            ctx.gbdtmo_partition_peer(p, lvl, self.state, self.xchg)
+            return
         if self.group is not None:
             parallel.exchange_keys(self.keys[: 1 << lvl], self.group)
         ctx.gbdtmo_split_record(p, lvl, self.ds.bins, self.dflt, self.q, self.scales, self.state, self.hist[cur],
@@ -258,6 +289,8 @@ class Booster:
                    n_rows=torch.empty(NH, dtype=torch.int64, device=dev),
                    n_left=torch.empty(NH, dtype=torch.int64, device=dev),
                    threshold=torch.empty(NH, dtype=torch.float32, device=dev))
+        # the current stream (after a graph capture the context still names the capture stream)
+        self.ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
         self.ctx.gbdtmo_tree_export(self.p, self.state, rec["node_state"], rec["feature"], rec["bin"], rec["gain"],
                                     rec["n_rows"], rec["n_left"], self.ds.cuts, rec["threshold"])
         if self.group is not None:   # thresholds live with the feature's owner: SUM merges them
@@ -291,7 +324,7 @@ class Booster:
 
 
 def train(X, Y, params: Params, device: str = "cuda:0", ctx: Optional[Context] = None, group=None,
-          f_begin: int = 0, m_global: Optional[int] = None):
+          f_begin: int = 0, m_global: Optional[int] = None, exchange: str = "collective"):
     """Public entry point: X float32 [n][m] and Y float32 [n][d] (host or device tensors or numpy
     arrays).  Copies the inputs to the GPU, bins the features, trains params.T trees, and
     returns the Booster (predictions in booster.pred, tree records in booster.trees)."""
@@ -303,7 +336,7 @@ def train(X, Y, params: Params, device: str = "cuda:0", ctx: Optional[Context] =
     Yd = Yt.to(dev, non_blocking=True).contiguous().float()
     ds = bin_features(ctx, Xd, params.B, f_begin=f_begin, m_global=m_global)
     del Xd
-    b = Booster(ctx, ds, Yd, params, group=group)
+    b = Booster(ctx, ds, Yd, params, group=group, exchange=exchange)
     b.fit()
     return b
 

@@ -2,6 +2,7 @@
 #include <new>
 
 #include "common.cuh"
+#include "peer.cuh"
 
 using namespace gbdtmo;
 
@@ -30,6 +31,7 @@ extern "C" gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out) {
 }
 
 extern "C" gbdtmo_status gbdtmo_destroy(gbdtmo_ctx c) {
+  if (c) peer_release((Ctx*)c);
   delete (Ctx*)c;
   return GBDTMO_OK;
 }
@@ -50,6 +52,10 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
     case GBDTMO_OPT_HIST_KERNEL:
       if (value < 0 || value > 2) { ctx->err = "gbdtmo_set_option: HIST_KERNEL must be 0, 1 or 2"; return GBDTMO_EINVAL; }
       ctx->hist_kernel = value;
+      return GBDTMO_OK;
+    case GBDTMO_OPT_PEER_TIMEOUT_MS:
+      if (value < 1) { ctx->err = "gbdtmo_set_option: PEER_TIMEOUT_MS must be >= 1"; return GBDTMO_EINVAL; }
+      ctx->peer_timeout_ms = value;
       return GBDTMO_OK;
     default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;
   }

@@ -14,6 +14,8 @@ namespace gbdtmo {
 
 // ------------------------------------------------------------------ context
 
+struct Peer;                   // peer-memory exchange group (peer.cu)
+
 struct Ctx {
   int device = 0;
   cudaStream_t stream = 0;
@@ -23,6 +25,8 @@ struct Ctx {
   int64_t gmem_max_rows = 0;   // GBDTMO_OPT_GMEM_MAX_ROWS: BUILD nodes with <= rows use the global-atomic variant
   int64_t small_max_rows = 0;  // GBDTMO_OPT_SMALL_MAX_ROWS: nodes whose parent's children both fit -> fused path
   int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16), 1 diagonal (K = 4), 2 TMA-staged row-pair
+  int64_t peer_timeout_ms = 30000;   // GBDTMO_OPT_PEER_TIMEOUT_MS: bound of every peer-flag wait
+  Peer* peer = nullptr;        // gbdtmo_peer_open / _connect (peer.cu)
   std::string err;
 };
 

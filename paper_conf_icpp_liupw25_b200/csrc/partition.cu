@@ -5,6 +5,7 @@
 // (bit = 1, left) and [begin + n_left, end) (right), both in their previous order, using a
 // global left-count prefix over positions (3 passes: tile counts, tile scan, scatter).
 #include "common.cuh"
+#include "peer.cuh"
 #include "plan.cuh"
 
 namespace gbdtmo {
@@ -12,7 +13,9 @@ namespace gbdtmo {
 // Apply the merged records: decisions for the level's nodes, child nodes, next-level plan.
 __global__ void __launch_bounds__(kPlanThreads)
 k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ xchg, int target_chunks,
-                int64_t gmem_max_rows, int64_t small_max_rows) {
+                int64_t gmem_max_rows, int64_t small_max_rows, uint64_t* __restrict__ peer_epoch) {
+  // peer exchange: both phases of this level are complete on this rank -> next epoch (peer.cuh)
+  if (peer_epoch && threadIdx.x == 0) *peer_epoch += 1;
   const int64_t LN = int64_t(1) << level, first = LN - 1;
   const int V = channels(p);
   const int64_t RW = rec_words(p);
@@ -200,6 +203,21 @@ k_part_scatter(gbdtmo_problem p, int level, State s, const int32_t* __restrict__
 
 using namespace gbdtmo;
 
+static gbdtmo_status partition_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t level, void* state,
+                                    const int64_t* xchg, uint64_t* peer_epoch) {
+  State s = state_view(*p, state);
+  const int64_t* bm = xchg + bitmap_offset(*p);
+  const int32_t* rows_in = (level & 1) ? s.rows1 : s.rows0;
+  int32_t* rows_out = (level & 1) ? s.rows0 : s.rows1;
+  const int64_t ntiles = part_tiles(*p);
+  GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p),
+            ctx->gmem_max_rows, small_rows(ctx, *p), peer_epoch);
+  GB_LAUNCH(k_part_count, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, bm);
+  GB_LAUNCH(k_part_scan, 1, kPartThreads, 0, ntiles, s);
+  GB_LAUNCH(k_part_scatter, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, rows_out, bm);
+  return GBDTMO_OK;
+}
+
 extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, void* state,
                                           const int64_t* xchg) {
   Ctx* ctx = (Ctx*)c;
@@ -208,15 +226,20 @@ extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p,
   GB_CHECK_ARG(!bad, bad ? bad : "");
   GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
   GB_CHECK_ARG(state && xchg, "null pointer");
-  State s = state_view(*p, state);
-  const int64_t* bm = xchg + bitmap_offset(*p);
-  const int32_t* rows_in = (level & 1) ? s.rows1 : s.rows0;
-  int32_t* rows_out = (level & 1) ? s.rows0 : s.rows1;
-  const int64_t ntiles = part_tiles(*p);
-  GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p),
-            ctx->gmem_max_rows, small_rows(ctx, *p));
-  GB_LAUNCH(k_part_count, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, bm);
-  GB_LAUNCH(k_part_scan, 1, kPartThreads, 0, ntiles, s);
-  GB_LAUNCH(k_part_scatter, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, rows_out, bm);
-  return GBDTMO_OK;
+  return partition_impl(ctx, p, level, state, xchg, nullptr);
+}
+
+extern "C" gbdtmo_status gbdtmo_partition_peer(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, void* state,
+                                               int64_t* xchg_merged) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  const char* bad = check_problem(p);
+  GB_CHECK_ARG(!bad, bad ? bad : "");
+  GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
+  GB_CHECK_ARG(state && xchg_merged, "null pointer");
+  GB_CHECK_ARG(peer_ready(ctx, *p), "peer group not connected for this problem shape (gbdtmo_peer_open/_connect)");
+  const gbdtmo_status st = peer_gather(ctx, *p, level, xchg_merged);
+  if (st != GBDTMO_OK) return st;
+  uint64_t* epoch = reinterpret_cast<uint64_t*>(peer_own_window(ctx)) + PEER_EPOCH;
+  return partition_impl(ctx, p, level, state, xchg_merged, epoch);
 }

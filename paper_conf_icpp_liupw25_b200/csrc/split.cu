@@ -5,7 +5,10 @@
 //   G_L^k, H_L^k, C_L = prefix sums over bins (exact int64 fixed point, MSE: H = 2 C),
 //   gain = 1/2 sum_k [G_L^2/(H_L+l) + G_R^2/(H_R+l) - G^2/(H+l)]   (Eq. 3, fp64),
 // valid iff C_L, C_R >= min_node; best per node by an atomicMax on a packed 64-bit key.
+#include <string.h>
+
 #include "common.cuh"
+#include "peer.cuh"
 
 namespace gbdtmo {
 
@@ -230,14 +233,37 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
                                const int64_t* __restrict__ hist,
                                const int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
                                const int32_t* __restrict__ pcnt, const uint64_t* __restrict__ keys,
-                               const float* __restrict__ scales, int64_t* __restrict__ xchg) {
+                               const float* __restrict__ scales, int64_t* __restrict__ xchg, PeerView pv,
+                               uint64_t* __restrict__ keys_merged) {
   const int slot = blockIdx.x;
   const int64_t h = (int64_t(1) << level) - 1 + slot;
   const int V = channels(p), B = p.B, m = p.m;
   const int64_t RW = rec_words(p);
   int64_t* rec = xchg + slot * RW;
+  uint64_t key;
+  if (pv.world > 0) {
+    // fused key exchange (peer.cuh): block 0 publishes this rank's keys, every block waits for the
+    // peers and takes the max of its slot's key over the N windows (= the MAX all-reduce)
+    __shared__ unsigned long long sk;
+    if (threadIdx.x == 0) {
+      const uint64_t E = peer_next_epoch(pv);
+      peer_publish_wait(pv, PEER_FLAG_KEYS, E, slot == 0);
+      const int64_t ko = peer_keys_off(p, level) / 8 + slot;
+      uint64_t k = 0;
+      for (int r = 0; r < pv.world; ++r) {
+        const uint64_t x = peer_load(reinterpret_cast<const uint64_t*>(pv.win[r]) + ko);
+        k = x > k ? x : k;
+      }
+      keys_merged[slot] = k;
+      sk = k;
+    }
+    __syncthreads();
+    key = sk;
+  } else {
+    key = keys[slot];
+  }
   int fl = 0, b = 0, fg = 0;
-  const bool own = s.node_state[h] == GBDTMO_NODE_ACTIVE && decode_local(p, keys[slot], &fl, &b, &fg);
+  const bool own = s.node_state[h] == GBDTMO_NODE_ACTIVE && decode_local(p, key, &fl, &b, &fg);
   if (!own) {
     for (int i = threadIdx.x; i < RW; i += blockDim.x) rec[i] = 0;
     return;
@@ -379,6 +405,23 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   return GBDTMO_OK;
 }
 
+static gbdtmo_status split_record_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t level, const uint8_t* bins,
+                                       const int32_t* dflt, const int32_t* q, const float* scales, void* state,
+                                       const int64_t* hist, const int32_t* cnt, const int64_t* parent_hist,
+                                       const int32_t* parent_cnt, const uint64_t* keys, int64_t* xchg,
+                                       const PeerView& pv, uint64_t* keys_merged) {
+  State s = state_view(*p, state);
+  const int64_t LN = int64_t(1) << level;
+  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, bins, q, s, hist, cnt, level > 0 ? parent_hist : hist,
+            level > 0 ? parent_cnt : cnt, keys, scales, xchg, pv, keys_merged);
+  // zero the record words of the unused slots of this buffer (levels < D-1) so SUM-merging is clean
+  const int64_t used = LN * rec_words(*p), cap = bitmap_offset(*p);
+  if (cap > used) GB_LAUNCH(k_zero_u64, 64, 256, 0, reinterpret_cast<uint64_t*>(xchg + used), cap - used);
+  GB_LAUNCH(k_bitmap, ctx->num_sms * 4, 256, (size_t)(2 * LN * sizeof(int)), *p, level, bins, s,
+            pv.world > 0 ? keys_merged : keys, xchg);
+  return GBDTMO_OK;
+}
+
 extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
                                              const uint8_t* bins, const int32_t* dflt, const int32_t* q,
                                              const float* scales, void* state,
@@ -392,13 +435,29 @@ extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem*
   GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
   GB_CHECK_ARG(bins && state && hist && cnt && keys && xchg && scales, "null pointer");
   GB_CHECK_ARG(level == 0 || (parent_hist && parent_cnt), "parent histogram required for level > 0");
-  State s = state_view(*p, state);
-  const int64_t LN = int64_t(1) << level;
-  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, bins, q, s, hist, cnt, level > 0 ? parent_hist : hist,
-            level > 0 ? parent_cnt : cnt, keys, scales, xchg);
-  // zero the record words of the unused slots of this buffer (levels < D-1) so SUM-merging is clean
-  const int64_t used = LN * rec_words(*p), cap = bitmap_offset(*p);
-  if (cap > used) GB_LAUNCH(k_zero_u64, 64, 256, 0, reinterpret_cast<uint64_t*>(xchg + used), cap - used);
-  GB_LAUNCH(k_bitmap, ctx->num_sms * 4, 256, (size_t)(2 * LN * sizeof(int)), *p, level, bins, s, keys, xchg);
-  return GBDTMO_OK;
+  PeerView none;
+  memset(&none, 0, sizeof(none));
+  return split_record_impl(ctx, p, level, bins, dflt, q, scales, state, hist, cnt, parent_hist, parent_cnt, keys, xchg,
+                           none, nullptr);
+}
+
+extern "C" gbdtmo_status gbdtmo_split_record_peer(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level,
+                                                  const uint8_t* bins, const int32_t* dflt, const int32_t* q,
+                                                  const float* scales, void* state,
+                                                  const int64_t* hist, const int32_t* cnt,
+                                                  const int64_t* parent_hist, const int32_t* parent_cnt,
+                                                  uint64_t* keys_merged) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  const char* bad = check_problem(p);
+  GB_CHECK_ARG(!bad, bad ? bad : "");
+  GB_CHECK_ARG(level >= 0 && level < p->D, "level out of range [0, D)");
+  GB_CHECK_ARG(bins && state && hist && cnt && keys_merged && scales, "null pointer");
+  GB_CHECK_ARG(level == 0 || (parent_hist && parent_cnt), "parent histogram required for level > 0");
+  GB_CHECK_ARG(peer_ready(ctx, *p), "peer group not connected for this problem shape (gbdtmo_peer_open/_connect)");
+  char* w = peer_own_window(ctx);
+  const uint64_t* keys = reinterpret_cast<const uint64_t*>(w + peer_keys_off(*p, level));
+  int64_t* xchg = reinterpret_cast<int64_t*>(w + peer_xchg_off(*p, level));
+  return split_record_impl(ctx, p, level, bins, dflt, q, scales, state, hist, cnt, parent_hist, parent_cnt, keys, xchg,
+                           peer_view(ctx), keys_merged);
 }

@@ -39,6 +39,11 @@ def test_sizes_and_validation_on_host():
     with pytest.raises(_abi.GbdtmoError):
         _abi.Context.gbdtmo_state_bytes(bad)
     assert _abi.Context.gbdtmo_bins_bytes(10, 16) == 10 * 16 + 32
+    # peer window (NEXT-4): header + per-level keys + per-level exchange buffers
+    xc = _abi.Context.gbdtmo_xchg_count(P)
+    wb = _abi.Context.gbdtmo_peer_window_bytes(P)
+    assert wb >= 512 + 8 * 8 * 128 + 8 * 8 * xc and wb < 512 + 8 * 8 * 128 + 8 * 8 * (xc + 32) + 256
+    assert _abi.Context.gbdtmo_peer_window_bytes(bad) == 0
 
 
 def test_create_without_gpu_fails_loudly():

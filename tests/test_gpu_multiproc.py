@@ -1,6 +1,9 @@
-"""The Booster's multi-rank path (feature shards + torch.distributed exchanges)
-run as two processes sharing cuda:0 over a gloo group: trees and predictions must equal the
-single-process run bit for bit.  (NCCL needs one GPU per rank; the exchange code is the same.)"""
+"""The Booster's multi-rank path (feature shards) run as two processes sharing cuda:0:
+trees and predictions must equal the single-process run bit for bit, for both exchanges —
+"collective" (torch.distributed all-reduces over a gloo group; NCCL needs one GPU per rank, the
+exchange code is the same) and "peer" (NEXT-4: the fused peer-memory exchange; the two processes'
+windows are mapped with CUDA IPC on the one device, the waits inside the kernels progress under
+the driver's time slicing between the two contexts).  The peer run also replays CUDA graphs."""
 import os
 import socket
 
@@ -27,7 +30,7 @@ def _case():
     return gen.WORKLOADS["C3"].scaled(n=60_000, m=30, T=2, D=5)
 
 
-def _worker(rank, world, port, out):
+def _worker(rank, world, port, out, exchange="collective", graph=False):
     import sys
     sys.path.insert(0, ROOT)
     import torch.distributed as dist
@@ -45,14 +48,25 @@ def _worker(rank, world, port, out):
     ds = pkg.bin_features(ctx, torch.from_numpy(np.ascontiguousarray(X[:, f0:f1])).cuda(), w.B, f_begin=f0,
                           m_global=w.m)
     P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).cuda(), P, group=dist.group.WORLD)
-    b.fit()
+    b = pkg.Booster(ctx, ds, torch.from_numpy(Y).cuda(), P, group=dist.group.WORLD, exchange=exchange)
+    if exchange == "peer":
+        ctx.gbdtmo_set_option(pkg._abi.OPT_PEER_TIMEOUT_MS, 120_000)
+    if graph:                         # trees replayed from one captured CUDA graph
+        b.capture()                   # (its warm-up runs one tree outside the graph: discarded)
+        b.pred.zero_()
+        b.trees.clear()
+        for _ in range(w.T):
+            b.step_graph()
+    else:
+        b.fit()
     torch.cuda.synchronize()
-    out[rank] = ([{k: v.cpu().numpy() for k, v in t.items()} for t in b.trees], b.pred.cpu().numpy())
+    status = b.peer_status() if exchange == "peer" else (0, 0)
+    out[rank] = ([{k: v.cpu().numpy() for k, v in t.items()} for t in b.trees], b.pred.cpu().numpy(), status)
     dist.destroy_process_group()
 
 
-def test_two_rank_booster_equals_single_rank():
+@pytest.mark.parametrize("exchange,graph", [("collective", False), ("peer", False), ("peer", True)])
+def test_two_rank_booster_equals_single_rank(exchange, graph):
     import sys
     sys.path.insert(0, ROOT)
     import paper_conf_icpp_liupw25_b200 as pkg
@@ -67,9 +81,12 @@ def test_two_rank_booster_equals_single_rank():
     torch.cuda.synchronize()
     mgr = mp.Manager()
     out = mgr.dict()
-    mp.start_processes(_worker, args=(2, _free_port(), out), nprocs=2, join=True, start_method="spawn")
+    mp.start_processes(_worker, args=(2, _free_port(), out, exchange, graph), nprocs=2, join=True, start_method="spawn")
     for rank in range(2):
-        trees, pred = out[rank]
+        trees, pred, (epoch, err) = out[rank]
+        assert err == 0, f"peer exchange error word {err:#x}"
+        if exchange == "peer":
+            assert epoch == (w.T + graph) * w.D          # one exchange per level (+ the capture warm-up tree)
         for t in range(w.T):
             a = {k: v.cpu().numpy() for k, v in ref.trees[t].items()}
             for k in ("node_state", "feature", "bin", "n_rows", "n_left", "leaf"):

@@ -385,6 +385,9 @@ def test_graph_replay_equals_eager(pkg, ctx):
         b.step_graph()
     torch.cuda.synchronize()
     assert torch.equal(a.pred, b.pred)
+    for ta, tb in zip(a.trees, b.trees):          # records exported after each replay
+        for k in ("node_state", "feature", "bin", "n_rows", "n_left", "leaf", "threshold"):
+            assert torch.equal(ta[k], tb[k]), k
 
 
 @pytest.mark.parametrize("case,sparse", [("C3s", False), ("C5s", False), ("C2s", True), ("C4s", False)])

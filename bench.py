@@ -356,6 +356,8 @@ def main():
                    "exchange": (exchange if world > 1 else "none") + (f" ({exchange_note})" if exchange_note else ""),
                    "l2": "inputs larger than L2", "graph": bool(a.graph and world == 1)},
         "hist_share": hist_total_ms / a.steps / ms_per_tree if ms_per_tree else None,
+        "hist_ms_by_level": ([round(float(np.mean(hist_ms[l::w.D])), 3) for l in range(w.D)]
+                             if len(hist_ms) == a.steps * w.D else None),
         "hist_rows_outputs_per_s_built": rows_built * w.d / (hist_total_ms * 1e-3) if hist_ms else None,
         "bin_ms": bin_ms, "bin_ms_first_call": bin_ms_first, "setup_s": setup_s,
         "roofline": {"bound": "alu", "kernel": "k_hist_smem (+k_zero_build) via gbdtmo_build_hist",

@@ -12,8 +12,10 @@
 //
 // E = epoch + 1, epoch = exchanges completed (a device word of the own window, incremented by the
 // partition's plan kernel), identical on every rank since all run the same sequence; CUDA graphs
-// replay correctly because nothing host-side carries the epoch.  Buffers are per level, so a rank
-// rewrites a buffer only after every peer has published a later flag, i.e. finished reading it.
+// replay correctly because nothing host-side carries the epoch.  A rank rewrites its keys only
+// after every peer published flag_rec (so finished reading them) and its records only after every
+// peer published the next flag_keys; one buffer per kind would be race-free, per-level buffers are
+// kept for debugging (model-checked: tests/test_peer_protocol.py).
 // Waits are bounded (GBDTMO_OPT_PEER_TIMEOUT_MS): on expiry the kernel records an error word
 // (gbdtmo_peer_status) and proceeds, so a lost peer cannot hang the GPU.
 #pragma once

@@ -11,6 +11,7 @@ from __future__ import annotations
 
 import dataclasses
 import math
+import os
 from typing import Optional
 
 import torch
@@ -210,6 +211,8 @@ class Booster:
         import torch.distributed as dist
         rank, world = dist.get_rank(self.group), dist.get_world_size(self.group)
         torch.cuda.synchronize(self.device)
+        if os.environ.get("GBDTMO_PEER_TIMEOUT_MS"):         # (tests: force expiry)
+            self.ctx.gbdtmo_set_option(_abi.OPT_PEER_TIMEOUT_MS, int(os.environ["GBDTMO_PEER_TIMEOUT_MS"]))
         h = self.ctx.gbdtmo_peer_open(self.p, rank, world)
         handles = [None] * world
         dist.all_gather_object(handles, h, group=self.group)

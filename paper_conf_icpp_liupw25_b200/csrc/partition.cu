@@ -13,9 +13,13 @@ namespace gbdtmo {
 // Apply the merged records: decisions for the level's nodes, child nodes, next-level plan.
 __global__ void __launch_bounds__(kPlanThreads)
 k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict__ xchg, int target_chunks,
-                int64_t gmem_max_rows, int64_t small_max_rows, uint64_t* __restrict__ peer_epoch) {
-  // peer exchange: both phases of this level are complete on this rank -> next epoch (peer.cuh)
-  if (peer_epoch && threadIdx.x == 0) *peer_epoch += 1;
+                int64_t gmem_max_rows, int64_t small_max_rows, uint64_t* __restrict__ peer_hdr) {
+  // peer exchange: both phases of this level are complete on this rank -> next epoch (peer.cuh).
+  // After an expired wait the merged records may be partial: no node splits (the tree ends in
+  // leaves, nothing is partitioned from inconsistent counts); the error stays recorded.
+  const bool peer_failed = peer_hdr && *reinterpret_cast<volatile uint64_t*>(peer_hdr + PEER_ERROR) != 0;
+  __syncthreads();
+  if (peer_hdr && threadIdx.x == 0) peer_hdr[PEER_EPOCH] += 1;
   const int64_t LN = int64_t(1) << level, first = LN - 1;
   const int V = channels(p);
   const int64_t RW = rec_words(p);
@@ -23,7 +27,7 @@ k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict_
     const int64_t h = first + i;
     if (s.node_state[h] != GBDTMO_NODE_ACTIVE) continue;
     const int64_t* rec = xchg + i * RW;
-    if (rec[V + 1] == 0) {                      // no valid split with gain > gamma: leaf
+    if (rec[V + 1] == 0 || peer_failed) {       // no valid split with gain > gamma: leaf
       s.node_state[h] = GBDTMO_NODE_LEAF;
       continue;
     }
@@ -193,7 +197,7 @@ k_part_scatter(gbdtmo_problem p, int level, State s, const int32_t* __restrict__
         dst = b + s.node_nleft[h] + (pos - b - lrank);
         s.nid[pi[i].r] = 2 * h + 2;
       }
-      rows_out[dst] = pi[i].r;
+      if (dst >= 0 && dst < p.n) rows_out[dst] = pi[i].r;   // (always true for consistent records)
     }
     excl += pi[i].left;
   }
@@ -204,14 +208,14 @@ k_part_scatter(gbdtmo_problem p, int level, State s, const int32_t* __restrict__
 using namespace gbdtmo;
 
 static gbdtmo_status partition_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t level, void* state,
-                                    const int64_t* xchg, uint64_t* peer_epoch) {
+                                    const int64_t* xchg, uint64_t* peer_hdr) {
   State s = state_view(*p, state);
   const int64_t* bm = xchg + bitmap_offset(*p);
   const int32_t* rows_in = (level & 1) ? s.rows1 : s.rows0;
   int32_t* rows_out = (level & 1) ? s.rows0 : s.rows1;
   const int64_t ntiles = part_tiles(*p);
   GB_LAUNCH(k_apply_records, 1, kPlanThreads, 0, *p, level, s, xchg, target_chunks_for(ctx, *p),
-            ctx->gmem_max_rows, small_rows(ctx, *p), peer_epoch);
+            ctx->gmem_max_rows, small_rows(ctx, *p), peer_hdr);
   GB_LAUNCH(k_part_count, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, bm);
   GB_LAUNCH(k_part_scan, 1, kPartThreads, 0, ntiles, s);
   GB_LAUNCH(k_part_scatter, (unsigned)ntiles, kPartThreads, 0, *p, level, s, rows_in, rows_out, bm);
@@ -240,6 +244,5 @@ extern "C" gbdtmo_status gbdtmo_partition_peer(gbdtmo_ctx c, const gbdtmo_proble
   GB_CHECK_ARG(peer_ready(ctx, *p), "peer group not connected for this problem shape (gbdtmo_peer_open/_connect)");
   const gbdtmo_status st = peer_gather(ctx, *p, level, xchg_merged);
   if (st != GBDTMO_OK) return st;
-  uint64_t* epoch = reinterpret_cast<uint64_t*>(peer_own_window(ctx)) + PEER_EPOCH;
-  return partition_impl(ctx, p, level, state, xchg_merged, epoch);
+  return partition_impl(ctx, p, level, state, xchg_merged, reinterpret_cast<uint64_t*>(peer_own_window(ctx)));
 }

@@ -84,11 +84,24 @@ __device__ inline bool peer_publish_wait(const PeerView& pv, int flag, uint64_t 
     const uint64_t* f = peer_word(pv, r, flag);
     while (peer_ld_acquire(f) < E) {
       if (peer_clock_ns() - t0 > (uint64_t)pv.timeout_ns) {
+        __threadfence_system();
         atomicCAS(reinterpret_cast<unsigned long long*>(peer_word(pv, pv.rank, PEER_ERROR)), 0ull,
                   (unsigned long long)(E << 8 | (uint64_t)(flag == PEER_FLAG_KEYS ? 1 : 2)));
         return false;
       }
       __nanosleep(128);
+    }
+  }
+  // a peer that failed earlier has diverged (its nodes became leaves): adopt its failure, so this
+  // rank stops splitting too instead of partitioning from records of a different tree.  The
+  // peer's error store precedes its flag store (fence), so the acquire above makes it visible.
+  for (int r = 0; r < pv.world; ++r) {
+    if (r == pv.rank) continue;
+    const uint64_t e = peer_ld_acquire(peer_word(pv, r, PEER_ERROR));
+    if (e) {
+      atomicCAS(reinterpret_cast<unsigned long long*>(peer_word(pv, pv.rank, PEER_ERROR)), 0ull,
+                (unsigned long long)e);
+      return false;
     }
   }
   return true;

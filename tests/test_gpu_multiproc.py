@@ -30,9 +30,11 @@ def _case():
     return gen.WORKLOADS["C3"].scaled(n=60_000, m=30, T=2, D=5)
 
 
-def _worker(rank, world, port, out, exchange="collective", graph=False):
+def _worker(rank, world, port, out, exchange="collective", graph=False, timeout_ms=None):
     import sys
     sys.path.insert(0, ROOT)
+    if timeout_ms is not None:
+        os.environ["GBDTMO_PEER_TIMEOUT_MS"] = str(timeout_ms)
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -49,7 +51,7 @@ def _worker(rank, world, port, out, exchange="collective", graph=False):
                           m_global=w.m)
     P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
     b = pkg.Booster(ctx, ds, torch.from_numpy(Y).cuda(), P, group=dist.group.WORLD, exchange=exchange)
-    if exchange == "peer":
+    if exchange == "peer" and timeout_ms is None:
         ctx.gbdtmo_set_option(pkg._abi.OPT_PEER_TIMEOUT_MS, 120_000)
     if graph:                         # trees replayed from one captured CUDA graph
         b.capture()                   # (its warm-up runs one tree outside the graph: discarded)
@@ -92,3 +94,25 @@ def test_two_rank_booster_equals_single_rank(exchange, graph):
             for k in ("node_state", "feature", "bin", "n_rows", "n_left", "leaf"):
                 np.testing.assert_array_equal(trees[t][k], a[k])
         np.testing.assert_array_equal(pred, ref.pred.cpu().numpy())
+
+
+def test_peer_wait_expiry_is_safe():
+    """Waits bounded at 1 ms (the two processes time-slice one GPU, so waits usually expire): the
+    run must finish without a fault, an expired wait is recorded in the error word, and every
+    level after it ends its nodes as leaves (no partition from partial records)."""
+    from gen import gen
+    w = _case()
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.start_processes(_worker, args=(2, _free_port(), out, "peer", False, 1), nprocs=2, join=True,
+                       start_method="spawn")
+    for rank in range(2):
+        trees, pred, (epoch, err) = out[rank]
+        assert np.all(np.isfinite(pred))
+        assert epoch == w.T * w.D
+        for t in trees:
+            st = t["node_state"]
+            assert set(np.unique(st)) <= {0, 1, 2}
+            assert t["n_rows"][0] == w.n and int(t["n_rows"][st == 2].sum()) == w.n   # leaves cover all rows
+        if err:
+            assert (err & 0xFF) in (1, 2)

@@ -66,6 +66,22 @@ def test_bin_matches_oracle(orc, pkg, ctx, case):
     np.testing.assert_array_equal(gb.T, bins)
 
 
+@pytest.mark.parametrize("case,strip", [("C1", 5), ("C3s", 8), ("C2s", 7)])
+def test_bin_host_strips_match_oracle(orc, pkg, ctx, case, strip):
+    """bin_features_host (column strips uploaded on a copy stream while the previous strip is
+    binned) gives the oracle's bins, cuts and nbins; ragged last strip."""
+    w = CASES[case]
+    X = gen.features_host(w)
+    Xh = torch.from_numpy(np.ascontiguousarray(X)).pin_memory()
+    ds = pkg.bin_features_host(ctx, Xh, w.B, DEV, strip=strip)
+    torch.cuda.synchronize()
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    np.testing.assert_array_equal(ds.nbins.cpu().numpy(), nbins)
+    np.testing.assert_array_equal(ds.cuts.cpu().numpy(), cuts)
+    gb = ds.bins[: w.n * ds.ld_bins].view(w.n, ds.ld_bins)[:, : w.m].cpu().numpy()
+    np.testing.assert_array_equal(gb.T, bins)
+
+
 def test_bin_edge_cases(orc, pkg, ctx):
     rng = np.random.default_rng(0)
     n = 9000

@@ -336,6 +336,8 @@ def main():
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except OSError:
         pass
+    hbm_peak = float(peaks.get("hbm_gbs") or 6650.0)      # B200_PROFILING.md fallback when the file is absent
+    hbm_peak_src = "MEASURED_PEAKS.json hbm_gbs" if peaks.get("hbm_gbs") else "of fallback (B200_PROFILING.md: 6.65 TB/s)"
     traffic = None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "hist_traffic.json")))
@@ -365,8 +367,8 @@ def main():
                      "frac": achieved / peak if peak else None, "traffic": traffic,
                      "peak_source": "guide: 32 banks x 4 B/clk/SM shared pipe -> 32 int32 ATOMS lanes/clk/SM, "
                                     "2 limbs per update, 148 SMs, 1.965 GHz max clock (DESIGN.md Roofline)",
-                     "hbm_view": {"achieved_gbs": hbm_gbs, "peak_gbs": peaks.get("hbm_gbs", 6553.6),
-                                  "frac": hbm_gbs / peaks.get("hbm_gbs", 6553.6)},
+                     "hbm_view": {"achieved_gbs": hbm_gbs, "peak_gbs": hbm_peak, "frac": hbm_gbs / hbm_peak,
+                                  "peak_source": hbm_peak_src},
                      "launches": hist_launches, "avg_launch_ms": hist_avg_ms},
         "clocks": clocks,
         "gpu_launches": int(l1 - l0),

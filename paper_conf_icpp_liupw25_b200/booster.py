@@ -271,10 +271,27 @@ class Booster:
         torch.cuda.synchronize(self.device)
         if os.environ.get("GBDTMO_PEER_TIMEOUT_MS"):         # (tests: force expiry)
             self.ctx.gbdtmo_set_option(_abi.OPT_PEER_TIMEOUT_MS, int(os.environ["GBDTMO_PEER_TIMEOUT_MS"]))
-        h = self.ctx.gbdtmo_peer_open(self.p, rank, world)
+        # every rank takes part in both gathers whatever happens locally, and all ranks agree on
+        # the outcome, so a failure anywhere raises everywhere (no rank left in a collective)
+        err = None
+        try:
+            h = self.ctx.gbdtmo_peer_open(self.p, rank, world)
+        except _abi.GbdtmoError as ex:
+            h, err = None, ex
         handles = [None] * world
         dist.all_gather_object(handles, h, group=self.group)
-        self.ctx.gbdtmo_peer_connect(b"".join(handles))
+        if err is None and all(x is not None for x in handles):
+            try:
+                self.ctx.gbdtmo_peer_connect(b"".join(handles))
+            except _abi.GbdtmoError as ex:
+                err = ex
+        elif err is None:
+            err = RuntimeError("gbdtmo_peer_open failed on another rank")
+        oks = [None] * world
+        dist.all_gather_object(oks, err is None, group=self.group)
+        if not all(oks):
+            self.ctx.gbdtmo_peer_close()
+            raise RuntimeError(f"peer exchange unavailable (rank {rank}: {err or 'ok'}; ranks ok: {oks})")
         self.peer_keys = [self.ctx.gbdtmo_peer_buffers(self.p, lvl)[0] for lvl in range(self.params.D)]
 
     def peer_status(self):

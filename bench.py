@@ -13,6 +13,7 @@ the device time per tree (max over ranks).  See DESIGN.md "Measurement".
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import subprocess
@@ -288,6 +289,10 @@ def main():
     clk = ClockSampler(local)
     clk.start()
     time.sleep(0.3)
+    # no Python GC pause inside the timed region (a gen-2 collection stalls the enqueueing thread
+    # for tens of ms and the GPU idles: measured as a run-to-run tail on the small configs)
+    gc.collect()
+    gc.disable()
     l0 = ctx.gbdtmo_launch_count()
     torch.cuda.synchronize()
     if group is not None:
@@ -301,6 +306,7 @@ def main():
             booster.step(time_hist=True)
     e1.record()
     torch.cuda.synchronize()
+    gc.enable()
     if group is not None:
         dist.barrier()
     l1 = ctx.gbdtmo_launch_count()
@@ -358,6 +364,8 @@ def main():
                    "exchange": (exchange if world > 1 else "none") + (f" ({exchange_note})" if exchange_note else ""),
                    "l2": "inputs larger than L2", "graph": bool(a.graph and world == 1)},
         "hist_share": hist_total_ms / a.steps / ms_per_tree if ms_per_tree else None,
+        "phase_ms_per_tree": ({k: round(v / a.steps, 3) for k, v in booster.phase_ms(a.steps).items()}
+                              if not (a.graph and world == 1) else None),
         "hist_ms_by_level": ([round(float(np.mean(hist_ms[l::w.D])), 3) for l in range(w.D)]
                              if len(hist_ms) == a.steps * w.D else None),
         "hist_rows_outputs_per_s_built": rows_built * w.d / (hist_total_ms * 1e-3) if hist_ms else None,
@@ -430,14 +438,16 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh, exchange="collecti
     ctx = pkg.Context(local)
     params = pkg.Params(loss=w.loss, T=a.steps, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
                         min_node=w.min_node)
+    pred_h = torch.empty((w.n, w.d), dtype=torch.float64, pin_memory=True)   # the caller's output buffer
     torch.cuda.synchronize()
     if group is not None:
         dist.barrier()
+    gc.collect()
+    gc.disable()
     e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
     e0.record()
     b = pkg.train(Xh, Yh, params, device=str(dev), ctx=ctx, group=group, f_begin=f0, m_global=w.m,
                   exchange=exchange)
-    pred_h = torch.empty(b.pred.shape, dtype=b.pred.dtype, pin_memory=True)
     pred_h.copy_(b.pred, non_blocking=True)
     model_bytes = 0
     for tr in b.trees:
@@ -446,6 +456,7 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh, exchange="collecti
     model_h = [{k: v.to("cpu", non_blocking=True) for k, v in tr.items()} for tr in b.trees]
     e1.record()
     torch.cuda.synchronize()
+    gc.enable()
     ms = e0.elapsed_time(e1)
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if group is not None:

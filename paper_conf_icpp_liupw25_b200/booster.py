@@ -262,6 +262,8 @@ class Booster:
         self.trees = []            # per tree: dict of device tensors (heap-indexed tree record)
         self._graph = None
         self.hist_events = []      # optional per-level (start, end) CUDA events around build_hist
+        self.phase_marks = []      # optional per-tree phase marks (time_hist=True), see phase_ms()
+        self._marks = []
 
     def _peer_connect(self):
         """Open this rank's window, exchange the IPC handles over the process group (plumbing),
@@ -315,15 +317,18 @@ class Booster:
         if time_hist:
             e1.record()
             self.hist_events.append((e0, e1))
+        self._mark("find_split", time_hist)
         peer = self.exchange == "peer"
         keys = self.peer_keys[lvl] if peer else self.keys     # peer: this level's window keys
         ctx.gbdtmo_find_split(p, lvl, self.ds.nbins, self.dflt, self.scales, self.state, self.hist[cur], self.cnt[cur],
                               ph, pc, keys)
         if self.small_max_rows > 0:
             ctx.gbdtmo_search_small(p, lvl, self.ds.bins, self.q, self.ds.nbins, self.scales, self.state, keys)
+        self._mark("split_record", time_hist)
         if peer:
             ctx.gbdtmo_split_record_peer(p, lvl, self.ds.bins, self.dflt, self.q, self.scales, self.state,
                                          self.hist[cur], self.cnt[cur], ph, pc, self.keys)
+            self._mark("partition", time_hist)
             ctx.gbdtmo_partition_peer(p, lvl, self.state, self.xchg)
             return
         if self.group is not None:
@@ -333,6 +338,7 @@ class Booster:
                                 ph, pc, self.keys, self.xchg)
         if self.group is not None:
             parallel.exchange_records(self.xchg, self.group)
+        self._mark("partition", time_hist)
         ctx.gbdtmo_partition(p, lvl, self.state, self.xchg)
 
     def _apply_options(self):
@@ -343,14 +349,36 @@ class Booster:
         ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_HIST_KERNEL, self.hist_kernel)
 
+    def _mark(self, name: str, on: bool):
+        """(timing) an event recorded before the phase `name`; the phase lasts until the next mark."""
+        if on:
+            e = torch.cuda.Event(enable_timing=True)
+            e.record()
+            self._marks.append((name, e))
+
+    def phase_ms(self, trees):
+        """Per-phase device ms summed over the last `trees` timed trees (from the marks)."""
+        tot = {}
+        for marks in self.phase_marks[-trees:]:
+            for (name, e0), (_, e1) in zip(marks[:-1], marks[1:]):
+                tot[name] = tot.get(name, 0.0) + e0.elapsed_time(e1)
+        return tot
+
     def _tree(self, time_hist: bool = False):
         ctx, p = self.ctx, self.p
         self._apply_options()
+        self._marks = []
+        self._mark("grad", time_hist)
         ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state)
         for lvl in range(self.params.D):
+            self._mark("build_hist", time_hist)
             self._level(lvl, time_hist)
+        self._mark("leaf+update", time_hist)
         ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf)
         ctx.gbdtmo_update_pred(p, self.state, self.leaf, self.pred)
+        self._mark("end", time_hist)
+        if time_hist:
+            self.phase_marks.append(self._marks)
 
     def step(self, time_hist: bool = False):
         """One boosting iteration (one tree) on the current stream; asynchronous."""

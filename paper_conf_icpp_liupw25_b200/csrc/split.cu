@@ -146,7 +146,33 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
 #pragma unroll
     for (int i = 0; i < kFsBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
     double P = 0.0;
+    // L2 prefetch of the channel rows GBDTMO_FS_PF channels ahead (softmax: g and h rows): the
+    // warp's loads are one dependent chain per channel, so without it ~55% of DRAM bandwidth
+    // is reached at this kernel's register-limited occupancy (ncu, profiles/r01f_ncu_fs_c5.txt)
+    auto prefetch = [&](int k) {
+      if (k >= V) return;
+      const int64_t o = (int64_t)k * B + lane * kFsBins;
+      if (derive) {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(phist + rowp + o));
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rows_ + o));
+      } else {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rowc + o));
+      }
+    };
+#ifndef GBDTMO_FS_PF
+#define GBDTMO_FS_PF 2
+#endif
+    constexpr int PF = GBDTMO_FS_PF;
+#pragma unroll
+    for (int k = 0; k < PF; ++k) {
+      prefetch(k);
+      if (SOFTMAX) prefetch(d + k);
+    }
     for (int k = 0; k < d; ++k) {
+      if (PF > 0) {
+        prefetch(k + PF);
+        if (SOFTMAX && k + PF < d) prefetch(d + k + PF);
+      }
       long long gv[kFsBins];
       int64_t* rg = hist + rowc + (int64_t)k * B;
       load_row8(gv, rg, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B, derive, store, B);

@@ -103,21 +103,26 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
              const float* __restrict__ scales, State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt,
              const int64_t* __restrict__ phist, const int32_t* __restrict__ pcnt,
              uint64_t* __restrict__ keys, int write_derived) {
-  const int slot = blockIdx.y;
+  // level 0: one node, warps = 8 features.  Deeper: a block holds a sibling pair, warps 0-3 the
+  // left child and 4-7 the right child over the same 4 features, so the derived child's reads
+  // of its built sibling's rows meet them in L2 while the sibling's own search streams them
+  // from DRAM (one DRAM pass over the built histogram instead of two).
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const bool paired = level > 0;
+  const int slot = paired ? 2 * blockIdx.y + (warp >> 2) : 0;
+  const int f = paired ? blockIdx.x * (kFsWarps / 2) + (warp & 3) : blockIdx.x * kFsWarps + warp;
   const int64_t h = (int64_t(1) << level) - 1 + slot;
-  if (s.node_state[h] != GBDTMO_NODE_ACTIVE || s.node_mode[h] == MODE_SMALL) return;   // SMALL: small.cu
+  const bool searched = s.node_state[h] == GBDTMO_NODE_ACTIVE && s.node_mode[h] != MODE_SMALL;  // SMALL: small.cu
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const bool store = derive && write_derived;
   const bool own = !derive || store;                  // this node's histogram may be written
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int f = blockIdx.x * kFsWarps + warp;
   const int sib = slot ^ 1, par = slot >> 1;
   const double lam = p.lambda;
   const int64_t* S = s.node_sum + h * (V + 1);         // exact node totals (channels, count)
   __shared__ unsigned long long wbest[kFsWarps];
   uint64_t best = 0;
-  if (f < m) {
+  if (searched && f < m) {
     const int db = dflt ? dflt[f] : -1;
     const int b0 = lane * kFsBins;
     // counts
@@ -231,9 +236,10 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   }
   if (lane == 0) wbest[warp] = best;
   __syncthreads();
-  if (threadIdx.x == 0) {
+  if (lane == 0 && (paired ? (warp & 3) == 0 : warp == 0)) {   // one reducer per slot in the block
+    const int w0 = paired ? warp : 0, nw = paired ? kFsWarps / 2 : kFsWarps;
     uint64_t bb = 0;
-    for (int w = 0; w < kFsWarps; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
+    for (int w = w0; w < w0 + nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
     if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
   }
 }
@@ -424,7 +430,8 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
-  dim3 grid((p->m + kFsWarps - 1) / kFsWarps, (unsigned)LN);
+  dim3 grid(level > 0 ? (p->m + kFsWarps / 2 - 1) / (kFsWarps / 2) : (p->m + kFsWarps - 1) / kFsWarps,
+            (unsigned)(level > 0 ? LN / 2 : 1));             // level > 0: sibling pairs (k_find_split)
   auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_find_split<true> : k_find_split<false>;
   GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, dflt, scales, s, hist, cnt,
             level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);

@@ -1,0 +1,13 @@
+# A/B: sibling-paired find_split blocks (current build) vs the previous build (build/ab/head)
+mkdir -p gpurun_out
+rm -f gpurun_out/abp_all.jsonl
+for rep in 1 2; do
+for lib in head def; do
+  if [ $lib = def ]; then L=""; else L="GBDTMO_LIB=build/ab/$lib/libgbdtmo.so"; fi
+  for wl in C2 S100 C4 C5; do
+    st=10; [ $wl = C5 ] && st=5
+    env $L timeout 400 python bench.py --workload $wl --no-e2e --no-cpu-baseline --steps $st --warmup 3 > gpurun_out/abp_${wl}_$lib.log 2>&1
+    (echo -n "$lib "; tail -1 gpurun_out/abp_${wl}_$lib.log) >> gpurun_out/abp_all.jsonl
+  done
+done
+done

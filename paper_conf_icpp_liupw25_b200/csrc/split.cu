@@ -13,6 +13,12 @@
 namespace gbdtmo {
 
 constexpr int kFsWarps = 8;      // warps per block = features of one node per block
+#ifndef GBDTMO_FS_PF
+#define GBDTMO_FS_PF 2           // channels of L2 prefetch ahead in the split search
+#endif
+#ifndef GBDTMO_FS_HALF
+#define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
+#endif
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 
 
@@ -164,9 +170,6 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
         asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rowc + o));
       }
     };
-#ifndef GBDTMO_FS_PF
-#define GBDTMO_FS_PF 2
-#endif
     constexpr int PF = GBDTMO_FS_PF;
 #pragma unroll
     for (int k = 0; k < PF; ++k) {
@@ -237,6 +240,225 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
   if (lane == 0) wbest[warp] = best;
   __syncthreads();
   if (lane == 0 && (paired ? (warp & 3) == 0 : warp == 0)) {   // one reducer per slot in the block
+    const int w0 = paired ? warp : 0, nw = paired ? kFsWarps / 2 : kFsWarps;
+    uint64_t bb = 0;
+    for (int w = w0; w < w0 + nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
+    if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
+  }
+}
+
+// Half-row variant (no default bins, 128 < B <= 256): two warps per (node, feature), lane l of
+// half h owns bins [128 h + 4 l, +4), so a lane holds half the row state of k_find_split and
+// the kernel runs at twice the occupancy (the 8-bin kernel is latency-bound at 128 registers:
+// ncu, profiles/r01g_ncu_fs_c2.txt).  The halves need no exchange: half 0 prefix-sums its
+// bins (left sums), half 1 suffix-sums its bins (right sums, bins > b) and both complete the
+// other side from the exact node totals (node_sum = the sum of the node's histogram row in
+// int64), so every G_L, G_R, C_L is the same integer as in k_find_split and the gains and
+// keys are bit-identical.
+constexpr int kFsHBins = 4;
+
+// half 0: inclusive prefix of 4 bins per lane over the warp; half 1: exclusive suffix (bins > b).
+__device__ __forceinline__ void half_scan(long long (&v)[kFsHBins], bool suffix) {
+  const int lane = threadIdx.x & 31;
+  if (!suffix) {
+#pragma unroll
+    for (int i = 1; i < kFsHBins; ++i) v[i] += v[i - 1];
+    long long tot;
+    const long long ex = warp_excl(v[kFsHBins - 1], &tot);
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) v[i] += ex;
+  } else {
+    long long run = 0;
+#pragma unroll
+    for (int i = kFsHBins - 1; i >= 0; --i) { const long long x = v[i]; v[i] = run; run += x; }
+    long long sfx = run;                                    // inclusive suffix over lanes
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long y = __shfl_down_sync(0xffffffffu, sfx, o);
+      if (lane + o < 32) sfx += y;
+    }
+    const long long ex = sfx - run;                         // lanes above this one
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) v[i] += ex;
+  }
+}
+
+// 4 consecutive bins [b0, b0 + 4) of one row (derived: parent - sibling, written back if store)
+__device__ __forceinline__ void load_row4(long long (&v)[kFsHBins], int b0, const int64_t* cur, const int64_t* par,
+                                          const int64_t* sib, bool derive, bool store, int B) {
+  if (b0 + kFsHBins <= B) {
+    if (derive) {
+      const longlong2* pp = reinterpret_cast<const longlong2*>(par + b0);
+      const longlong2* ps = reinterpret_cast<const longlong2*>(sib + b0);
+      const longlong2 a0 = pp[0], a1 = pp[1], c0 = ps[0], c1 = ps[1];
+      const longlong2 x0 = make_longlong2(a0.x - c0.x, a0.y - c0.y), x1 = make_longlong2(a1.x - c1.x, a1.y - c1.y);
+      if (store) {
+        longlong2* pc = reinterpret_cast<longlong2*>(const_cast<int64_t*>(cur) + b0);
+        pc[0] = x0; pc[1] = x1;
+      }
+      v[0] = x0.x; v[1] = x0.y; v[2] = x1.x; v[3] = x1.y;
+    } else {
+      const longlong2* pc = reinterpret_cast<const longlong2*>(cur + b0);
+      const longlong2 x0 = pc[0], x1 = pc[1];
+      v[0] = x0.x; v[1] = x0.y; v[2] = x1.x; v[3] = x1.y;
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) {
+      const int b = b0 + i;
+      long long x = 0;
+      if (b < B) {
+        if (derive) { x = par[b] - sib[b]; if (store) const_cast<int64_t*>(cur)[b] = x; }
+        else x = cur[b];
+      }
+      v[i] = x;
+    }
+  }
+}
+
+template <bool SOFTMAX>
+#ifndef GBDTMO_FS_HMINB
+#define GBDTMO_FS_HMINB 3        // resident blocks per SM the half-row kernel is compiled for
+#endif
+__global__ void __launch_bounds__(kFsWarps * 32, GBDTMO_FS_HMINB)
+k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
+               State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
+               const int32_t* __restrict__ pcnt, uint64_t* __restrict__ keys, int write_derived) {
+  // warps: [sibling (paired levels: warp >> 2)][feature][half]; level 0: [feature (4)][half]
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int half = warp & 1;
+  const bool paired = level > 0;
+  const int slot = paired ? 2 * blockIdx.y + (warp >> 2) : 0;
+  const int f = paired ? blockIdx.x * 2 + ((warp >> 1) & 1) : blockIdx.x * 4 + (warp >> 1);
+  const int64_t h = (int64_t(1) << level) - 1 + slot;
+  const bool searched = s.node_state[h] == GBDTMO_NODE_ACTIVE && s.node_mode[h] != MODE_SMALL;
+  const bool derive = s.node_mode[h] == MODE_DERIVE;
+  const bool store = derive && write_derived;
+  const int V = channels(p), B = p.B, m = p.m, d = p.d;
+  const int sib = slot ^ 1, par = slot >> 1;
+  const double lam = p.lambda;
+  const int64_t* S = s.node_sum + h * (V + 1);
+  __shared__ unsigned long long wbest[kFsWarps];
+  uint64_t best = 0;
+  const int b0 = half * (32 * kFsHBins) + lane * kFsHBins;
+  if (searched && f < m && half * (32 * kFsHBins) < B) {
+    // counts -> C_L per bin
+    long long cl[kFsHBins];
+    const long long ctot = S[V];
+    {
+      const int64_t oc = ((int64_t)slot * m + f) * B, os = ((int64_t)sib * m + f) * B, op = ((int64_t)par * m + f) * B;
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) {
+        const int b = b0 + i;
+        long long x = 0;
+        if (b < B) {
+          if (derive) { x = pcnt[op + b] - cnt[os + b]; if (store) cnt[oc + b] = (int32_t)x; }
+          else x = cnt[oc + b];
+        }
+        cl[i] = x;
+      }
+      half_scan(cl, half);
+      if (half) {
+#pragma unroll
+        for (int i = 0; i < kFsHBins; ++i) cl[i] = ctot - cl[i];
+      }
+    }
+    const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
+                  rowp = ((int64_t)par * m + f) * V * B;
+    double accL[kFsHBins], accR[kFsHBins];
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
+    double P = 0.0;
+    auto prefetch = [&](int k) {
+      if (k >= V) return;
+      const int64_t o = (int64_t)k * B + b0;
+      if (derive) {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(phist + rowp + o));
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rows_ + o));
+      } else {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rowc + o));
+      }
+    };
+    constexpr int PF = GBDTMO_FS_PF;
+#pragma unroll
+    for (int k = 0; k < PF; ++k) {
+      prefetch(k);
+      if (SOFTMAX) prefetch(d + k);
+    }
+    for (int k = 0; k < d; ++k) {
+      if (PF > 0) {
+        prefetch(k + PF);
+        if (SOFTMAX && k + PF < d) prefetch(d + k + PF);
+      }
+      // left sums GL[i] and right sums G - GL[i] as exact integers
+      long long gl[kFsHBins];
+      load_row4(gl, b0, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
+                derive, store, B);
+      half_scan(gl, half);
+      const long long G = S[k];
+      if (half) {
+#pragma unroll
+        for (int i = 0; i < kFsHBins; ++i) gl[i] = G - gl[i];
+      }
+      const double sg = (double)scales[k];
+      if (!SOFTMAX) {
+#pragma unroll
+        for (int i = 0; i < kFsHBins; ++i) {
+          const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
+          accL[i] = fma(GL, GL, accL[i]);
+          accR[i] = fma(GR, GR, accR[i]);
+        }
+        const double Gd = (double)G * sg;
+        P = fma(Gd, Gd, P);
+      } else {
+        long long hl[kFsHBins];
+        load_row4(hl, b0, hist + rowc + (int64_t)(d + k) * B, phist + rowp + (int64_t)(d + k) * B,
+                  hist + rows_ + (int64_t)(d + k) * B, derive, store, B);
+        half_scan(hl, half);
+        const long long H = S[d + k];
+        if (half) {
+#pragma unroll
+          for (int i = 0; i < kFsHBins; ++i) hl[i] = H - hl[i];
+        }
+        const double sh = (double)scales[d + k];
+#pragma unroll
+        for (int i = 0; i < kFsHBins; ++i) {
+          const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
+          const double HL = (double)hl[i] * sh, HR = (double)(H - hl[i]) * sh;
+          accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+        }
+        const double Gd = (double)G * sg, Hd = (double)H * sh;
+        P += Gd * Gd / (Hd + lam);
+      }
+    }
+    const int nb = nbins[f];
+    const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) {
+      const int b = b0 + i;
+      const long long c = cl[i];
+      if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
+        double gain;
+        if (!SOFTMAX)
+          gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
+                        P / (2.0 * (double)ctot + lam));
+        else
+          gain = 0.5 * (accL[i] - P);
+        if (gain > p.gamma) {
+          const uint64_t key = pack_split_key(gain, fb0 + b);
+          best = key > best ? key : best;
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
+    best = y > best ? y : best;
+  }
+  if (lane == 0) wbest[warp] = best;
+  __syncthreads();
+  if (lane == 0 && (paired ? (warp & 3) == 0 : warp == 0)) {
     const int w0 = paired ? warp : 0, nw = paired ? kFsWarps / 2 : kFsWarps;
     uint64_t bb = 0;
     for (int w = w0; w < w0 + nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
@@ -430,9 +652,18 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
+  const bool softmax = p->loss == GBDTMO_LOSS_SOFTMAX;
+  if (GBDTMO_FS_HALF && !dflt && p->B > 128) {
+    // two warps per (node, feature): 2 features x 2 siblings per block, level 0: 4 features
+    dim3 grid(level > 0 ? (p->m + 1) / 2 : (p->m + 3) / 4, (unsigned)(level > 0 ? LN / 2 : 1));
+    auto kern = softmax ? k_find_split_h<true> : k_find_split_h<false>;
+    GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt, level > 0 ? parent_hist : hist,
+              level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
+    return GBDTMO_OK;
+  }
   dim3 grid(level > 0 ? (p->m + kFsWarps / 2 - 1) / (kFsWarps / 2) : (p->m + kFsWarps - 1) / kFsWarps,
             (unsigned)(level > 0 ? LN / 2 : 1));             // level > 0: sibling pairs (k_find_split)
-  auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_find_split<true> : k_find_split<false>;
+  auto kern = softmax ? k_find_split<true> : k_find_split<false>;
   GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, dflt, scales, s, hist, cnt,
             level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
   return GBDTMO_OK;

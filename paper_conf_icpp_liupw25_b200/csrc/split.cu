@@ -20,6 +20,7 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
 #endif
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
+constexpr int kRecChannels = 64; // record channels per k_split_record block
 
 
 // Exclusive prefix (over lanes) and total of a per-lane int64.
@@ -494,6 +495,8 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   const int V = channels(p), B = p.B, m = p.m;
   const int64_t RW = rec_words(p);
   int64_t* rec = xchg + slot * RW;
+  // blockIdx.y: block of kRecChannels channels of the record (c = V is the count)
+  const int c0 = blockIdx.y * kRecChannels, c1 = min(V + 1, c0 + kRecChannels);
   uint64_t key;
   if (pv.world > 0) {
     // fused key exchange (peer.cuh): block 0 publishes this rank's keys, every block waits for the
@@ -501,14 +504,14 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
     __shared__ unsigned long long sk;
     if (threadIdx.x == 0) {
       const uint64_t E = peer_next_epoch(pv);
-      peer_publish_wait(pv, PEER_FLAG_KEYS, E, slot == 0);
+      peer_publish_wait(pv, PEER_FLAG_KEYS, E, slot == 0 && blockIdx.y == 0);
       const int64_t ko = peer_keys_off(p, level) / 8 + slot;
       uint64_t k = 0;
       for (int r = 0; r < pv.world; ++r) {
         const uint64_t x = peer_load(reinterpret_cast<const uint64_t*>(pv.win[r]) + ko);
         k = x > k ? x : k;
       }
-      keys_merged[slot] = k;
+      if (blockIdx.y == 0) keys_merged[slot] = k;
       sk = k;
     }
     __syncthreads();
@@ -519,7 +522,8 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   int fl = 0, b = 0, fg = 0;
   const bool own = s.node_state[h] == GBDTMO_NODE_ACTIVE && decode_local(p, key, &fl, &b, &fg);
   if (!own) {
-    for (int i = threadIdx.x; i < RW; i += blockDim.x) rec[i] = 0;
+    for (int i = c0 + threadIdx.x; i < c1; i += blockDim.x) rec[i] = 0;
+    if (blockIdx.y == 0 && threadIdx.x < 3) rec[V + 1 + threadIdx.x] = 0;
     return;
   }
   const bool derive = s.node_mode[h] == MODE_DERIVE;
@@ -529,6 +533,7 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   const int db = dflt ? dflt[fl] : -1;            // default bin: recovered from the node totals
   const int64_t* S = s.node_sum + h * (V + 1);
   if (s.node_mode[h] == MODE_SMALL) {             // not materialised: left sums straight from the rows
+    if (blockIdx.y != 0) return;                  // (d <= 32: one block covers every channel)
     // one pass: warps take 32 rows at a time, lanes = channels sum the rows that go left
     __shared__ long long acc[2 * 32 + 1];
     for (int c = threadIdx.x; c <= V; c += blockDim.x) acc[c] = 0;
@@ -556,7 +561,7 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
     __syncthreads();
     for (int c = threadIdx.x; c <= V; c += blockDim.x) rec[c] = acc[c];
   } else
-  for (int c = warp; c <= V; c += nw) {           // c == V: the counts
+  for (int c = c0 + warp; c < c1; c += nw) {      // c == V: the counts
     long long le = 0, all = 0;
     for (int bb = lane; bb < B; bb += 32) {
       if (bb == db) continue;
@@ -575,31 +580,44 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
     if (db >= 0 && db <= b) le += S[c] - all;      // (S[V] = the node's row count)
     if (lane == 0) rec[c] = le;
   }
-  if (threadIdx.x == 0) {
+  if (blockIdx.y == 0 && threadIdx.x == 0) {
     rec[V + 1] = fg + 1;
     rec[V + 2] = b;
   }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    // exact Eq. (3) at the winner from the exact sums (informational: the tree record's gain)
-    const int d = p.d;
-    const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
-    const long long ctot = S[V], cl = rec[V];
-    double g = 0.0;
-    for (int k = 0; k < d; ++k) {
-      const double sg = (double)scales[k];
-      const double GL = (double)rec[k] * sg, G = (double)S[k] * sg, GR = (double)(S[k] - rec[k]) * sg;
-      double HL, H, HR;
-      if (softmax) {
-        const double sh = (double)scales[d + k];
-        HL = (double)rec[d + k] * sh; H = (double)S[d + k] * sh; HR = (double)(S[d + k] - rec[d + k]) * sh;
-      } else {
-        HL = 2.0 * cl; H = 2.0 * ctot; HR = 2.0 * (ctot - cl);
-      }
-      g += GL * GL / (HL + p.lambda) + GR * GR / (HR + p.lambda) - G * G / (H + p.lambda);
+}
+
+// Exact Eq. (3) at each owned winner from the record's exact left sums (informational: the tree
+// record's gain; the choice was made on the keys).  One warp per slot, lanes over outputs.
+__global__ void k_record_gain(gbdtmo_problem p, int level, State s, const float* __restrict__ scales,
+                              int64_t* __restrict__ xchg) {
+  const int lane = threadIdx.x & 31;
+  const int64_t slot = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t LN = int64_t(1) << level;
+  if (slot >= LN) return;
+  const int V = channels(p), d = p.d;
+  const int64_t RW = rec_words(p);
+  int64_t* rec = xchg + slot * RW;
+  if (rec[V + 1] == 0) return;                   // not split here / not owned by this rank
+  const int64_t h = LN - 1 + slot;
+  const int64_t* S = s.node_sum + h * (V + 1);
+  const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
+  const long long ctot = S[V], cl = rec[V];
+  double g = 0.0;
+  for (int k = lane; k < d; k += 32) {
+    const double sg = (double)scales[k];
+    const double GL = (double)rec[k] * sg, G = (double)S[k] * sg, GR = (double)(S[k] - rec[k]) * sg;
+    double HL, H, HR;
+    if (softmax) {
+      const double sh = (double)scales[d + k];
+      HL = (double)rec[d + k] * sh; H = (double)S[d + k] * sh; HR = (double)(S[d + k] - rec[d + k]) * sh;
+    } else {
+      HL = 2.0 * cl; H = 2.0 * ctot; HR = 2.0 * (ctot - cl);
     }
-    rec[V + 3] = __double_as_longlong(0.5 * g);
+    g += GL * GL / (HL + p.lambda) + GR * GR / (HR + p.lambda) - G * G / (H + p.lambda);
   }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) g += __shfl_xor_sync(0xffffffffu, g, o);
+  if (lane == 0) rec[V + 3] = __double_as_longlong(0.5 * g);
 }
 
 // Row-direction bitmap (owner's bits only): bit i = instance i is in a splitting node of this
@@ -676,8 +694,10 @@ static gbdtmo_status split_record_impl(Ctx* ctx, const gbdtmo_problem* p, int32_
                                        const PeerView& pv, uint64_t* keys_merged) {
   State s = state_view(*p, state);
   const int64_t LN = int64_t(1) << level;
-  GB_LAUNCH(k_split_record, (unsigned)LN, 256, 0, *p, level, dflt, bins, q, s, hist, cnt, level > 0 ? parent_hist : hist,
-            level > 0 ? parent_cnt : cnt, keys, scales, xchg, pv, keys_merged);
+  const unsigned cb = (unsigned)((channels(*p) + 1 + kRecChannels - 1) / kRecChannels);
+  GB_LAUNCH(k_split_record, dim3((unsigned)LN, cb), 256, 0, *p, level, dflt, bins, q, s, hist, cnt,
+            level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, scales, xchg, pv, keys_merged);
+  GB_LAUNCH(k_record_gain, (unsigned)((LN + 7) / 8), 256, 0, *p, level, s, scales, xchg);
   // zero the record words of the unused slots of this buffer (levels < D-1) so SUM-merging is clean
   const int64_t used = LN * rec_words(*p), cap = bitmap_offset(*p);
   if (cap > used) GB_LAUNCH(k_zero_u64, 64, 256, 0, reinterpret_cast<uint64_t*>(xchg + used), cap - used);

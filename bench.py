@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--graph", action="store_true", help="replay each tree as a CUDA graph (1 GPU)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N > 1 (gloo: lets N ranks share one GPU for testing)")
+    ap.add_argument("--no-root-cache", action="store_true", help="(A/B) accumulate the root counts every tree")
     ap.add_argument("--exchange", default="auto", choices=["auto", "peer", "collective"],
                     help="N > 1 split exchange: peer = fused peer-memory exchange inside the kernels (NEXT-4), "
                          "collective = torch.distributed all-reduces; auto = peer, verified after the warm-up "
@@ -256,7 +257,8 @@ def main():
     exchange = a.exchange if a.exchange != "auto" else ("peer" if world > 1 else "collective")
     exchange_note = None
     try:
-        booster = pkg.Booster(ctx, ds, Y, params, group=group, exchange=exchange)
+        booster = pkg.Booster(ctx, ds, Y, params, group=group, exchange=exchange,
+                              cache_root_counts=not a.no_root_cache)
     except Exception as ex:            # e.g. CUDA IPC unavailable: the collective path
         if a.exchange == "peer":
             raise

@@ -115,6 +115,14 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
 enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3,
        GBDTMO_OPT_PEER_TIMEOUT_MS = 4 /* bound of every peer-flag wait (gbdtmo_peer_*), default 30000 */ };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
+/* Cached root counts.  The root holds all n rows in every tree, so its count histogram
+ * cnt[0][f][b] = #{i : bin(i, f) = b} (PAPER.md:214's histogram, count channel) is the same for
+ * every tree of a dataset.  root_cnt: int32 [m][B] device, e.g. a copy of the level-0 `cnt` of
+ * the first tree (after gbdtmo_find_split, which completes default-bin counts); owned by the
+ * caller, must stay valid while set; NULL (default) disables.  While set, gbdtmo_build_hist at
+ * level 0 copies it into `cnt` and skips the count accumulation (not with histogram kernel 2 or
+ * when the root would use the global-atomic variant).  Results are identical. */
+gbdtmo_status gbdtmo_set_root_counts(gbdtmo_ctx ctx, const int32_t* root_cnt);
 /* Number of kernels this context has launched so far (for launch accounting). */
 int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
 

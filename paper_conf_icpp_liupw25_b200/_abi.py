@@ -28,7 +28,7 @@ SYMBOLS = (
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
     "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
     "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
-    "gbdtmo_partition_peer",
+    "gbdtmo_partition_peer", "gbdtmo_set_root_counts",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS = 1, 2, 3, 4
 PEER_HANDLE_BYTES = 64
@@ -91,6 +91,7 @@ def lib():
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_predict": ([P, P, i64, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
             "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
+            "gbdtmo_set_root_counts": ([P, P], C.c_int),
             "gbdtmo_peer_window_bytes": ([PP], sz),
             "gbdtmo_peer_open": ([P, PP, i32, i32, P], C.c_int),
             "gbdtmo_peer_connect": ([P, P], C.c_int),
@@ -147,6 +148,9 @@ class Context:
 
     def gbdtmo_set_option(self, option: int, value: int):
         self._check(lib().gbdtmo_set_option(self._h, option, value), "gbdtmo_set_option")
+
+    def gbdtmo_set_root_counts(self, root_cnt):
+        self._check(lib().gbdtmo_set_root_counts(self._h, _ptr(root_cnt)), "gbdtmo_set_root_counts")
 
     def gbdtmo_launch_count(self) -> int:
         return int(lib().gbdtmo_launch_count(self._h))

@@ -196,7 +196,7 @@ class Booster:
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
                  small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
-                 packed_bins: Optional[bool] = None, exchange: str = "collective"):
+                 packed_bins: Optional[bool] = None, exchange: str = "collective", cache_root_counts: bool = True):
         """exchange (only with `group`): "collective" = torch.distributed all-reduces per level;
         "peer" = the fused peer-memory exchange (NEXT-4, gbdtmo_*_peer): the keys / records are
         read from the other ranks' windows inside split_record / partition, no host collective."""
@@ -252,6 +252,9 @@ class Booster:
             ctx.gbdtmo_pack_bins(self.p, ds.bins, self.packed)
         self.keys = torch.zeros(1 << max(D - 1, 0), dtype=torch.int64, device=dev)
         self.xchg = torch.zeros(ctx.gbdtmo_xchg_count(self.p), dtype=torch.int64, device=dev)
+        # root counts are the same for every tree (all rows): cached after the first tree's level 0
+        self.cache_root_counts = cache_root_counts
+        self.root_cnt = None
         self.peer_keys = None
         if self.exchange == "peer":
             self._peer_connect()
@@ -348,6 +351,7 @@ class Booster:
         ctx.gbdtmo_set_option(_abi.OPT_GMEM_MAX_ROWS, self.gmem_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_HIST_KERNEL, self.hist_kernel)
+        ctx.gbdtmo_set_root_counts(self.root_cnt)
 
     def _mark(self, name: str, on: bool):
         """(timing) an event recorded before the phase `name`; the phase lasts until the next mark."""
@@ -373,6 +377,9 @@ class Booster:
         for lvl in range(self.params.D):
             self._mark("build_hist", time_hist)
             self._level(lvl, time_hist)
+            if lvl == 0 and self.cache_root_counts and self.root_cnt is None:
+                # (plumbing: one device copy per dataset) the level-0 counts after find_split
+                self.root_cnt = self.cnt[0][: self.p.m * self.p.B].clone()
         self._mark("leaf+update", time_hist)
         ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf)
         ctx.gbdtmo_update_pred(p, self.state, self.leaf, self.pred)

@@ -27,6 +27,7 @@ struct Ctx {
   int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16), 1 diagonal (K = 4), 2 TMA-staged row-pair
   int64_t peer_timeout_ms = 30000;   // GBDTMO_OPT_PEER_TIMEOUT_MS: bound of every peer-flag wait
   Peer* peer = nullptr;        // gbdtmo_peer_open / _connect (peer.cu)
+  const int32_t* root_cnt = nullptr;   // gbdtmo_set_root_counts: cached root counts [m][B] (or null)
   std::string err;
 };
 
@@ -92,6 +93,7 @@ struct HistCfg {
   int n_ct;   // channel tiles
   int n_ft;   // feature tiles
   int smem;   // bytes of dynamic shared memory
+  int no_cnt; // 1: counts come from the cached root counts (gbdtmo_set_root_counts), not accumulated
 };
 
 #ifndef GBDTMO_HIST_LCNT
@@ -121,6 +123,7 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
   c.smem = k * limbs_per_feature + 4 * hist_cnt_words(c.K, k, p.B) + kHistWarps * 32 * 8 * ((k + 7) / 8);
+  c.no_cnt = 0;
   return c;
 }
 
@@ -241,7 +244,8 @@ inline const char* check_problem(const gbdtmo_problem* p) {
 // The diagonal shared-memory histogram variant (hist_diag.cu).
 HistCfg hist_config_diag(const gbdtmo_problem& p);
 gbdtmo_status launch_hist_diag(Ctx* ctx, const gbdtmo_problem& p, const uint8_t* bins, const int32_t* q,
-                               const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt);
+                               const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt,
+                               bool no_cnt);
 // The TMA-staged shared-memory histogram variant (hist_tma.cu).
 bool hist_tma_supported(const gbdtmo_problem& p, const uint8_t* bins);
 HistCfg hist_config_tma(const gbdtmo_problem& p, int max_smem);

@@ -104,7 +104,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int f0 = ft * KF;
     const int kk = min(KF, m - f0);
     const int c0 = ct * K;
-    const bool do_cnt = (ct == 0);
+    const bool do_cnt = (ct == 0) && !hc.no_cnt;
     int dfl[KF];                                   // default (skipped) bin per feature, -1: none
 #pragma unroll
     for (int j = 0; j < KF; ++j) dfl[j] = (SKIP && j < kk) ? __ldg(&dflt[f0 + j]) : -1;
@@ -351,11 +351,18 @@ k_hist_gmem(gbdtmo_problem p, const uint8_t* __restrict__ bins, const int32_t* _
   }
 }
 
-// Zero the histogram slots of the level's BUILD nodes (the flush accumulates atomically).
+// Zero the histogram slots of the level's BUILD nodes (the flush accumulates atomically).  With
+// cached root counts (level 0), the root's count slot is filled from the cache instead (the
+// histogram kernels then skip the count atomics), whatever the root's build mode.
 __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __restrict__ hist,
-                             int32_t* __restrict__ cnt) {
+                             int32_t* __restrict__ cnt, const int32_t* __restrict__ root_cnt) {
   const int64_t slot = blockIdx.y;
   const int64_t h = (int64_t(1) << level) - 1 + slot;
+  if (root_cnt) {
+    const int64_t cw = (int64_t)p.m * p.B;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += (int64_t)gridDim.x * blockDim.x)
+      cnt[i] = root_cnt[i];
+  }
   if (s.node_mode[h] != MODE_BUILD) return;
   const int64_t V = channels(p);
   const int64_t hw = (int64_t)p.m * p.B * V;           // int64 words per slot
@@ -368,7 +375,8 @@ __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __re
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < hv; i += stride)
     reinterpret_cast<longlong2*>(hb)[i] = make_longlong2(0, 0);
   for (int64_t i = 2 * hv + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < hw; i += stride) hb[i] = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += stride) cb[i] = 0;
+  if (!root_cnt)
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cw; i += stride) cb[i] = 0;
 }
 
 template <int K, int KF, bool SKIP, bool PACKED>
@@ -443,15 +451,19 @@ gbdtmo_status build_hist_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t level, 
   State s = state_view(*p, state);
   HistCfg hc = hist_config(*p);
   const int64_t LN = int64_t(1) << level;
+  // cached root counts: level 0, a variant that can skip its counts, and no global-atomic root
+  const bool tma = ctx->hist_kernel == 2 && !dflt && hist_tma_supported(*p, bins);
+  const int32_t* root_cnt = (level == 0 && ctx->root_cnt && !tma && ctx->gmem_max_rows < p->n) ? ctx->root_cnt : nullptr;
+  hc.no_cnt = root_cnt ? 1 : 0;
   int gx = (int)(2 * ctx->num_sms / (LN > 1 ? LN / 2 : 1));
   if (gx < 8) gx = 8;
-  GB_LAUNCH(k_zero_build, dim3(gx, (unsigned)LN), 256, 0, *p, level, s, hist, cnt);
+  GB_LAUNCH(k_zero_build, dim3(gx, (unsigned)LN), 256, 0, *p, level, s, hist, cnt, root_cnt);
   const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
   const int use_rows = level > 0;
   gbdtmo_status st;
   if (ctx->hist_kernel == 1 && !dflt) {
-    st = launch_hist_diag(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
-  } else if (ctx->hist_kernel == 2 && !dflt && hist_tma_supported(*p, bins)) {
+    st = launch_hist_diag(ctx, *p, bins, q, rows, use_rows, s, hist, cnt, root_cnt != nullptr);
+  } else if (tma) {
     st = launch_hist_tma(ctx, *p, bins, q, rows, use_rows, s, hist, cnt);
   } else switch (hc.K) {
     case 4: st = launch_hist<4>(ctx, *p, hc, bins, packed, dflt, q, rows, use_rows, s, hist, cnt); break;
@@ -512,5 +524,12 @@ extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p,
   GB_CHECK_ARG(hist_packable(*p), "feature tiles wider than 8 features: no packed layout (gbdtmo_packed_bins_bytes = 0)");
   const HistCfg hc = hist_config(*p);
   GB_LAUNCH(k_pack_bins, ctx->num_sms * 8, 256, 0, *p, hc.k, hc.n_ft, bins, reinterpret_cast<uint64_t*>(packed));
+  return GBDTMO_OK;
+}
+
+extern "C" gbdtmo_status gbdtmo_set_root_counts(gbdtmo_ctx c, const int32_t* root_cnt) {
+  Ctx* ctx = (Ctx*)c;
+  if (!ctx) return GBDTMO_EINVAL;
+  ctx->root_cnt = root_cnt;
   return GBDTMO_OK;
 }

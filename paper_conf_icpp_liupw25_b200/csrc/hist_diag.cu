@@ -34,6 +34,7 @@ HistCfg hist_config_diag(const gbdtmo_problem& p) {
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
   c.smem = k * per_feature + kHistWarps * 32 * 4 * (k / 4 + 1);
+  c.no_cnt = 0;
   return c;
 }
 
@@ -98,7 +99,7 @@ k_hist_diag(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     const int f0 = ft * KF;
     const int kk = min(KF, m - f0);
     const int c0 = ct * K;
-    const bool do_cnt = (ct == 0);
+    const bool do_cnt = (ct == 0) && !hc.no_cnt;
     for (int i = threadIdx.x * 4; i < limb_words; i += blockDim.x * 4)
       *reinterpret_cast<uint4*>(&sm[i]) = make_uint4(0, 0, 0, 0);
     for (int i = limb_words + threadIdx.x; i < limb_words + cnt_words; i += blockDim.x) sm[i] = 0;
@@ -238,8 +239,10 @@ static gbdtmo_status launch_diag_kf(Ctx* ctx, const gbdtmo_problem& p, const His
 }
 
 gbdtmo_status launch_hist_diag(Ctx* ctx, const gbdtmo_problem& p, const uint8_t* bins, const int32_t* q,
-                               const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
-  const HistCfg hc = hist_config_diag(p);
+                               const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt,
+                               bool no_cnt) {
+  HistCfg hc = hist_config_diag(p);
+  hc.no_cnt = no_cnt ? 1 : 0;
   switch (hc.k) {
     case 20: return launch_diag_kf<20>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);
     case 16: return launch_diag_kf<16>(ctx, p, hc, bins, q, rows, use_rows, s, hist, cnt);

@@ -60,6 +60,7 @@ HistCfg hist_config_tma(const gbdtmo_problem& p, int max_smem) {
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
   c.smem = k * per_feature + tma_fixed_bytes(p.B);
+  c.no_cnt = 0;
   return c;
 }
 

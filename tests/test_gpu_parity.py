@@ -406,6 +406,31 @@ def test_graph_replay_equals_eager(pkg, ctx):
             assert torch.equal(ta[k], tb[k]), k
 
 
+@pytest.mark.parametrize("case,sparse,kernel", [("C3s", False, None), ("C2s", True, None), ("C2s", False, 1),
+                                               ("C1", False, None)])
+def test_cached_root_counts_equal_accumulated(pkg, ctx, case, sparse, kernel):
+    """gbdtmo_set_root_counts: trees 2.. take the root's count histogram from the cache instead of
+    accumulating it; trees, leaves and predictions are identical (both shared-memory variants and
+    the sparsity-aware path, where find_split completes the cached default-bin counts)."""
+    w = CASES[case]
+    X, Y = _inputs(w)
+    P = _params(pkg, w, T=3)
+    out = []
+    for cache in (False, True):
+        ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
+        b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), P, sparse_default=sparse, hist_kernel=kernel,
+                        cache_root_counts=cache)
+        b.fit()
+        torch.cuda.synchronize()
+        assert (b.root_cnt is not None) == cache
+        out.append(b)
+    a, c = out
+    assert torch.equal(a.pred, c.pred)
+    for ta, tc in zip(a.trees, c.trees):
+        for k in ("node_state", "feature", "bin", "n_rows", "n_left", "leaf"):
+            assert torch.equal(ta[k], tc[k]), k
+
+
 @pytest.mark.parametrize("case,sparse", [("C3s", False), ("C5s", False), ("C2s", True), ("C4s", False)])
 def test_packed_bins_layout_and_equivalence(orc, pkg, ctx, case, sparse):
     """gbdtmo_pack_bins writes the documented [tile][row][8] layout (checked against a numpy

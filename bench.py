@@ -130,6 +130,23 @@ def built_rows(tree_np, D):
     return total
 
 
+def built_rows_by_level(tree_np, D):
+    """Rows built per level (level 0: the root; level l+1: smaller children of level-l splits)."""
+    st, nr, nl = tree_np["node_state"], tree_np["n_rows"], tree_np["n_left"]
+    out = [0] * D
+    if st[0] in (1, 2) and tree_np["_searched"].get(0, False):
+        out[0] = int(nr[0])
+    for h in range(len(st)):
+        if st[h] == 1:
+            lvl = int(np.floor(np.log2(h + 1)))
+            if lvl + 1 >= D:
+                continue
+            l, r = 2 * h + 1, 2 * h + 2
+            if tree_np["_searched"].get(l, False) or tree_np["_searched"].get(r, False):
+                out[lvl + 1] += int(min(nl[h], nr[h] - nl[h]))
+    return out
+
+
 def annotate_searched(tree_np, D, min_node):
     st, nr = tree_np["node_state"], tree_np["n_rows"]
     s = {}
@@ -368,6 +385,7 @@ def main():
         "hist_share": hist_total_ms / a.steps / ms_per_tree if ms_per_tree else None,
         "phase_ms_per_tree": ({k: round(v / a.steps, 3) for k, v in booster.phase_ms(a.steps).items()}
                               if not (a.graph and world == 1) else None),
+        "rows_built_by_level": [int(np.mean([built_rows_by_level(tr, w.D)[l] for tr in trees])) for l in range(w.D)],
         "hist_ms_by_level": ([round(float(np.mean(hist_ms[l::w.D])), 3) for l in range(w.D)]
                              if len(hist_ms) == a.steps * w.D else None),
         "hist_rows_outputs_per_s_built": rows_built * w.d / (hist_total_ms * 1e-3) if hist_ms else None,

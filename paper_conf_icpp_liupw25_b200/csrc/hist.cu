@@ -62,6 +62,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #ifndef GBDTMO_HIST_SB
 #define GBDTMO_HIST_SB 8
 #endif
+#ifndef GBDTMO_HIST_WDEPTH
+#define GBDTMO_HIST_WDEPTH 1       // batches of bin-window prefetch (2: A/B for gathered levels)
+#endif
 #ifndef GBDTMO_HIST_SHFL
 #define GBDTMO_HIST_SHFL 0         // (A/B) 1: phase 2 takes the bins by SHFL, no scratch round trip
 #endif
@@ -145,14 +148,26 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
     };
     int r_cur = load_rid(beg + warp * 32 + lane);
     int r_nxt = load_rid(beg + warp * 32 + bstep + lane);
+#if GBDTMO_HIST_WDEPTH == 2
+    int r_n2 = load_rid(beg + warp * 32 + 2 * bstep + lane);
+    uint64_t w_n1[NW];
+    load_win(r_nxt, w_n1);
+#endif
     uint64_t w_cur[NW];
     load_win(r_cur, w_cur);
     int qv[SB];
     load_q(r_cur, 0, qv);
     for (int b0 = beg + warp * 32; b0 < end; b0 += bstep) {
+#if GBDTMO_HIST_WDEPTH == 2
+      // (gathered deep levels) bin windows two batches ahead, row ids three
+      const int r_n3 = load_rid(b0 + 3 * bstep + lane);
+      uint64_t w_n2[NW];
+      load_win(r_n2, w_n2);
+#else
       const int r_nn = load_rid(b0 + 2 * bstep + lane);
       uint64_t w_nxt[NW];
       load_win(r_nxt, w_nxt);
+#endif
       // ---- phase 1: lane l owns row b0 + l (invalid rows: window 0, q 0, not counted)
       const int r = r_cur;
       uint64_t sw[SW];
@@ -223,10 +238,18 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         for (int t = 0; t < SB; ++t) qv[t] = qn[t];
       }
       __syncwarp();
+#if GBDTMO_HIST_WDEPTH == 2
+      r_cur = r_nxt;
+      r_nxt = r_n2;
+      r_n2 = r_n3;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) { w_cur[i] = w_n1[i]; w_n1[i] = w_n2[i]; }
+#else
       r_cur = r_nxt;
       r_nxt = r_nn;
 #pragma unroll
       for (int i = 0; i < NW; ++i) w_cur[i] = w_nxt[i];
+#endif
     }
     __syncthreads();
 

@@ -60,7 +60,7 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #define GBDTMO_HIST_NOCOUNT 0      // (experiment only: drops the counts; results invalid)
 #endif
 #ifndef GBDTMO_HIST_SB
-#define GBDTMO_HIST_SB 8
+#define GBDTMO_HIST_SB 2          // q-prefetch groups: 2 keeps the batch loop spill-free at 64 registers (8 spilled: C5 -10%)
 #endif
 #ifndef GBDTMO_HIST_WDEPTH
 #define GBDTMO_HIST_WDEPTH 1       // batches of bin-window prefetch (2: A/B for gathered levels)

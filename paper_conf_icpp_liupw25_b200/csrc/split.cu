@@ -319,9 +319,12 @@ __device__ __forceinline__ void load_row4(long long (&v)[kFsHBins], int b0, cons
 
 template <bool SOFTMAX>
 #ifndef GBDTMO_FS_HMINB
-#define GBDTMO_FS_HMINB 3        // resident blocks per SM the half-row kernel is compiled for
+#define GBDTMO_FS_HMINB 3        // resident blocks per SM the half-row kernel is compiled for (MSE)
 #endif
-__global__ void __launch_bounds__(kFsWarps * 32, GBDTMO_FS_HMINB)
+#ifndef GBDTMO_FS_HMINB_SOFTMAX
+#define GBDTMO_FS_HMINB_SOFTMAX 4   // (softmax: 4 measured faster on C2 / C4-shaped rows despite spills)
+#endif
+__global__ void __launch_bounds__(kFsWarps * 32, SOFTMAX ? GBDTMO_FS_HMINB_SOFTMAX : GBDTMO_FS_HMINB)
 k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
                State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
                const int32_t* __restrict__ pcnt, uint64_t* __restrict__ keys, int write_derived) {

@@ -322,7 +322,7 @@ template <bool SOFTMAX>
 #define GBDTMO_FS_HMINB 3        // resident blocks per SM the half-row kernel is compiled for (MSE)
 #endif
 #ifndef GBDTMO_FS_HMINB_SOFTMAX
-#define GBDTMO_FS_HMINB_SOFTMAX 4   // (softmax: 4 measured faster on C2 / C4-shaped rows despite spills)
+#define GBDTMO_FS_HMINB_SOFTMAX 3   // (4: C2 find_split 2.51 -> 2.34 ms but S500 3.0 -> 5.5 ms: spills at d = 500)
 #endif
 __global__ void __launch_bounds__(kFsWarps * 32, SOFTMAX ? GBDTMO_FS_HMINB_SOFTMAX : GBDTMO_FS_HMINB)
 k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,

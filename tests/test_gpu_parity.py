@@ -406,6 +406,30 @@ def test_graph_replay_equals_eager(pkg, ctx):
             assert torch.equal(ta[k], tb[k]), k
 
 
+@pytest.mark.parametrize("case", ["C1", "C3s", "C2s"])
+def test_public_train_from_host_matches_oracle(orc, pkg, ctx, case):
+    """The public entry point bench.py's e2e leg times: pkg.train() from pinned HOST X / Y (strip
+    upload overlapped with binning, then the trees): trees equal the oracle's, predictions within
+    the north star's 1e-4."""
+    w = CASES[case]
+    X, Y = _inputs(w)
+    Xh = torch.from_numpy(np.ascontiguousarray(X)).pin_memory()
+    Yh = torch.from_numpy(np.ascontiguousarray(Y)).pin_memory()
+    P = _params(pkg, w)
+    b = pkg.train(Xh, Yh, P, device=DEV, ctx=ctx)
+    torch.cuda.synchronize()
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    for t in range(w.T):
+        st = b.trees[t]["node_state"].cpu().numpy()
+        assert np.array_equal(st, ref["state"][t]), t
+        split = st == 1
+        assert np.array_equal(b.trees[t]["feature"].cpu().numpy()[split], ref["feat"][t][split])
+        assert np.array_equal(b.trees[t]["bin"].cpu().numpy()[split], ref["bin"][t][split])
+    assert np.max(np.abs(b.pred.cpu().numpy() - ref["pred"])) < 1e-4
+
+
 @pytest.mark.parametrize("case,sparse,kernel", [("C3s", False, None), ("C2s", True, None), ("C2s", False, 1),
                                                ("C1", False, None)])
 def test_cached_root_counts_equal_accumulated(pkg, ctx, case, sparse, kernel):

@@ -51,7 +51,10 @@ struct Ctx {
 // ----------------------------------------------------------------- constants
 
 constexpr int kQShift = 30;            // q = rint(g * 2^30 / P), |q| <= 2^30
-constexpr int kChunkMax = 65536;       // rows per histogram work item: lo-limb sums < 2^32
+#ifndef GBDTMO_CHUNK_MAX
+#define GBDTMO_CHUNK_MAX 65536
+#endif
+constexpr int kChunkMax = GBDTMO_CHUNK_MAX;   // rows per histogram work item: lo-limb sums < 2^32 (<= 65536)
 constexpr int kChunkMin = 512;
 constexpr int kPartTile = 2048;        // positions per partition block
 #ifndef GBDTMO_HIST_THREADS

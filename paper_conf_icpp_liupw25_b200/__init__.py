@@ -2,3 +2,4 @@
 subtraction and multi-output split search behind the C ABI of include/gbdtmo.h."""
 from ._abi import Context, Problem, GbdtmoError, LOSS_MSE, LOSS_SOFTMAX, lib  # noqa: F401
 from .booster import Params, Dataset, Booster, bin_features, bin_features_host, bin_features_csc, train, predict  # noqa: F401
+from . import parallel  # noqa: F401

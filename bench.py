@@ -373,7 +373,7 @@ def main():
     traffic = None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "hist_traffic.json")))
-        if prof.get("workload") == w.name:
+        if prof.get("workload") == w.name and world == 1:     # (captured on one GPU, all features)
             traffic = prof.get("dram_bytes_per_launch")
     except (OSError, ValueError):
         pass

@@ -62,6 +62,9 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #ifndef GBDTMO_HIST_SB
 #define GBDTMO_HIST_SB 2          // q-prefetch groups: 2 keeps the batch loop spill-free at 64 registers (8 spilled: C5 -10%)
 #endif
+#ifndef GBDTMO_HIST_MATCHCNT
+#define GBDTMO_HIST_MATCHCNT 0     // (A/B) 1: counts combined across lanes with MATCH.ANY
+#endif
 #ifndef GBDTMO_HIST_WDEPTH
 #define GBDTMO_HIST_WDEPTH 1       // batches of bin-window prefetch (2: A/B for gathered levels)
 #endif
@@ -182,12 +185,22 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
             sw[i] = keep >= 8 ? sw[i] : keep <= 0 ? 0ull : (sw[i] & ((1ull << (8 * keep)) - 1));
           }
         }
-        if (!LCNT && do_cnt && !GBDTMO_HIST_NOCOUNT) {
+        if (!LCNT && do_cnt && !GBDTMO_HIST_NOCOUNT && !GBDTMO_HIST_MATCHCNT) {
 #pragma unroll
           for (int j = 0; j < KF; ++j) {         // features j >= kk land in slots never flushed
             const uint32_t bin = byte_of<SW>(sw, j);
             if (!SKIP || (int)bin != dfl[j]) red_shared_add(acnt + 4u * (j * B + bin), 1u);  // counts[j][b]
           }
+        }
+      }
+      if (GBDTMO_HIST_MATCHCNT && !LCNT && do_cnt && !GBDTMO_HIST_NOCOUNT) {
+        // (A/B) lanes with equal bins combine first: one atomic per distinct bin (MATCH.ANY)
+#pragma unroll
+        for (int j = 0; j < KF; ++j) {
+          const uint32_t bin = byte_of<SW>(sw, j);
+          const bool on = r >= 0 && (!SKIP || (int)bin != dfl[j]);
+          const unsigned peers = __match_any_sync(0xffffffffu, on ? bin : 0x100u + lane);
+          if (on && lane == __ffs(peers) - 1) red_shared_add(acnt + 4u * (j * B + bin), (uint32_t)__popc(peers));
         }
       }
 #pragma unroll

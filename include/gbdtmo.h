@@ -377,6 +377,10 @@ gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx ctx, const uint8_t* handles /* host
 gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level,
                                   uint64_t** keys /* host out */, int64_t** xchg /* host out */);
 gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx ctx, int64_t* epoch /* host */, int64_t* error /* host */);
+/* gbdtmo_peer_status_async: the same two words (epoch, error) copied asynchronously on the
+ *   context's stream into out[0], out[1] (int64; pinned host or device memory, caller-owned), so
+ *   a driver can check the error word once per tree without a device synchronisation. */
+gbdtmo_status gbdtmo_peer_status_async(gbdtmo_ctx ctx, int64_t* out /* 2 words */);
 gbdtmo_status gbdtmo_peer_close(gbdtmo_ctx ctx);
 /* gbdtmo_split_record with the key exchange fused in: keys are read from every window (no
  * `keys` argument), records and bitmap go to the own window (no `xchg` argument); keys_merged

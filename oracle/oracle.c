@@ -243,6 +243,30 @@ void oracle_update_pred(double* pred, int32_t d, const int32_t* rows, int64_t nr
     for (int32_t k = 0; k < d; ++k) pred[(int64_t)rows[t] * d + k] += v[k];
 }
 
+/* ------------------------------------------------------------- inference */
+
+/* Tree walk for unseen rows (see oracle.h).  The split test is bin(x) <= b with
+ * bin(x) = #{cuts <= x} (R14, R15), evaluated from the raw feature value. */
+void oracle_predict(const float* X, int64_t n, int64_t ld_x, const float* cuts, const int32_t* nbins,
+                    int32_t B, int32_t T, int32_t D, int32_t d, const int32_t* state,
+                    const int32_t* feat, const int32_t* bin, const double* leaf, double* pred) {
+  const int64_t slots = ((int64_t)1 << (D + 1)) - 1;
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < n; ++i) {
+    for (int32_t t = 0; t < T; ++t) {
+      const int32_t* st = state + (int64_t)t * slots;
+      int64_t h = 0;
+      while (h < slots && st[h] == 1) {
+        const int32_t f = feat[(int64_t)t * slots + h];
+        const int32_t b = count_cuts_le(cuts + (int64_t)f * (B - 1), nbins[f] - 1, X[i * ld_x + f]);
+        h = (b <= bin[(int64_t)t * slots + h]) ? 2 * h + 1 : 2 * h + 2;
+      }
+      if (h < slots && st[h] == 2)
+        for (int32_t k = 0; k < d; ++k) pred[i * d + k] += leaf[((int64_t)t * slots + h) * d + k];
+    }
+  }
+}
+
 /* ----------------------------------------------------------- Algorithm 1 */
 
 static void node_totals(const double* g, const double* h, int32_t d, const int32_t* rows,

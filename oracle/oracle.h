@@ -29,6 +29,8 @@
  *   oracle_train (MSE)    pinned  (sklearn residual-tree boosting, λ=0)
  *   oracle_train (softmax) pinned  (d = 2: sklearn HistGradientBoostingClassifier, binary log loss;
  *                                   d > 2: per-step pins only)
+ *   oracle_predict        pinned  (on the training rows = oracle_train's incremental prediction,
+ *                                   a different computation; sklearn tree.predict on unseen rows)
  */
 #ifndef GBDTMO_ORACLE_H
 #define GBDTMO_ORACLE_H
@@ -119,6 +121,17 @@ void oracle_train(const uint16_t* bins_cm, int64_t n, int32_t m, const int32_t* 
                   double* pred,
                   int32_t* state, int32_t* feat, int32_t* bin, double* gain, int64_t* n_left,
                   int64_t* nrows, double* leaf);
+
+/* Inference for (unseen) instances ("predictions" for new data; the traversal the
+ * training path avoids).  For every row i and tree t = 0..T-1 in order: start at the
+ * root (heap id 0); at a split node (state 1) go to child 2h+1 iff bin(X[i][feat], cuts of feat)
+ * <= bin (the split's own definition, R14 + R15: left = {bin <= b}), else 2h+2; at a leaf
+ * (state 2) add leaf[t][h][0..d) to pred[i].  X row-major [n][ld_x] (raw features), cuts
+ * [m][B-1] from oracle_bin, state/feat/bin int32 [T][NH], leaf fp64 [T][NH][d] as written by
+ * oracle_train (NH = 2^(D+1) - 1); pred [n][d] in/out. */
+void oracle_predict(const float* X, int64_t n, int64_t ld_x, const float* cuts, const int32_t* nbins,
+                    int32_t B, int32_t T, int32_t D, int32_t d, const int32_t* state,
+                    const int32_t* feat, const int32_t* bin, const double* leaf, double* pred);
 
 /* Number of worker threads the oracle uses (OpenMP), for reporting. */
 int32_t oracle_num_threads(void);

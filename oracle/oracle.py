@@ -58,6 +58,7 @@ def lib():
         _LIB.oracle_update_pred.argtypes = [P, i32, P, i64, P]
         _LIB.oracle_train.argtypes = [P, i64, i32, P, i32, P, i32, C.POINTER(Params), P,
                                       P, P, P, P, P, P, P]
+        _LIB.oracle_predict.argtypes = [P, i64, i64, P, P, i32, i32, i32, i32, P, P, P, P, P]
         _LIB.oracle_num_threads.restype = i32
     return _LIB
 
@@ -186,3 +187,18 @@ def train(bins_cm, nbins, B, y, loss=LOSS_MSE, T=5, D=4, lam=1.0, gamma=0.0, lr=
                        _p(state), _p(feat), _p(binv), _p(gain_), _p(n_left), _p(nrows), _p(leaf))
     return dict(pred=pred, state=state, feat=feat, bin=binv, gain=gain_, n_left=n_left,
                 nrows=nrows, leaf=leaf)
+
+
+def predict(X, cuts, nbins, B, ref, D, T=None, pred=None):
+    """Tree walk over raw features (oracle_predict) with the trees of an
+    oracle.train result `ref` (its first T trees); returns pred [n][d] fp64."""
+    X = _c(X, np.float32); cuts = _c(cuts, np.float32); nbins = _c(nbins, np.int32)
+    n = X.shape[0]
+    T = ref["state"].shape[0] if T is None else T
+    d = ref["leaf"].shape[2]
+    st = _c(ref["state"][:T], np.int32); ft = _c(ref["feat"][:T], np.int32); bt = _c(ref["bin"][:T], np.int32)
+    lf = _c(ref["leaf"][:T], np.float64)
+    pred = np.zeros((n, d)) if pred is None else _c(pred, np.float64).copy()
+    lib().oracle_predict(_p(X), n, X.shape[1], _p(cuts), _p(nbins), B, T, D, d, _p(st), _p(ft), _p(bt), _p(lf),
+                         _p(pred))
+    return pred

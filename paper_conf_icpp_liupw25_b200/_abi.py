@@ -28,7 +28,7 @@ SYMBOLS = (
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
     "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
     "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
-    "gbdtmo_partition_peer", "gbdtmo_set_root_counts",
+    "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS = 1, 2, 3, 4
 PEER_HANDLE_BYTES = 64
@@ -98,6 +98,7 @@ def lib():
             "gbdtmo_peer_buffers": ([P, PP, i32, C.POINTER(P), C.POINTER(P)], C.c_int),
             "gbdtmo_peer_status": ([P, C.POINTER(i64), C.POINTER(i64)], C.c_int),
             "gbdtmo_peer_close": ([P], C.c_int),
+            "gbdtmo_peer_status_async": ([P, P], C.c_int),
             "gbdtmo_split_record_peer": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_partition_peer": ([P, PP, i32, P, P], C.c_int),
         }
@@ -286,6 +287,9 @@ class Context:
         e, r = C.c_int64(), C.c_int64()
         self._check(lib().gbdtmo_peer_status(self._h, C.byref(e), C.byref(r)), "gbdtmo_peer_status")
         return int(e.value), int(r.value)
+
+    def gbdtmo_peer_status_async(self, out):
+        self._check(lib().gbdtmo_peer_status_async(self._h, _ptr(out)), "gbdtmo_peer_status_async")
 
     def gbdtmo_peer_close(self):
         self._check(lib().gbdtmo_peer_close(self._h), "gbdtmo_peer_close")

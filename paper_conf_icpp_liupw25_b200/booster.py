@@ -63,6 +63,11 @@ def variant_threshold(V: int, m: int, key: str = "gmem_max_rows", n: Optional[in
     return int(e.get(key, 0))
 
 
+class PeerExchangeError(RuntimeError):
+    """A bounded peer-flag wait of the fused exchange expired (gbdtmo_peer_status error word != 0):
+    the trees trained since are not valid (every later node becomes a leaf)."""
+
+
 def _align(x, a):
     return (x + a - 1) // a * a
 
@@ -256,6 +261,8 @@ class Booster:
         self.cache_root_counts = cache_root_counts
         self.root_cnt = None
         self.peer_keys = None
+        self._peer_host = None          # pinned int64 [2]: (epoch, error) copied after every tree
+        self._peer_evt = None
         if self.exchange == "peer":
             self._peer_connect()
         NH = (1 << (D + 1)) - 1
@@ -302,6 +309,34 @@ class Booster:
     def peer_status(self):
         """(exchanges completed, error word) of the peer window (synchronous); error 0 = healthy."""
         return self.ctx.gbdtmo_peer_status()
+
+    def check_peer(self, block: bool = False):
+        """Raise PeerExchangeError if the peer window's (sticky) error word is set.  Reads the
+        copy enqueued after the last tree (gbdtmo_peer_status_async); block=False only looks if
+        that copy has landed (no device synchronisation), block=True waits for it."""
+        if self._peer_evt is None:
+            return
+        if not block and not self._peer_evt.query():
+            return
+        self._peer_evt.synchronize()
+        epoch, err = int(self._peer_host[0]), int(self._peer_host[1])
+        if err:
+            raise PeerExchangeError(
+                f"peer exchange wait expired (error word {err:#x}: epoch {err >> 8}, phase {err & 0xFF}; "
+                f"{epoch} exchanges completed): trees trained since then are invalid")
+
+    def _peer_after_tree(self):
+        """Once per tree, asynchronously: check the previous tree's status copy if it has landed,
+        then enqueue a copy of this tree's (epoch, error) words (no host synchronisation)."""
+        if self.exchange != "peer":
+            return
+        self.check_peer(block=False)
+        if self._peer_host is None:
+            self._peer_host = torch.zeros(2, dtype=torch.int64).pin_memory()
+        self.ctx.gbdtmo_set_stream(torch.cuda.current_stream(self.device).cuda_stream)
+        self.ctx.gbdtmo_peer_status_async(self._peer_host)
+        self._peer_evt = torch.cuda.Event()
+        self._peer_evt.record(torch.cuda.current_stream(self.device))
 
     # ------------------------------------------------------------------ one tree
     def _level(self, lvl: int, time_hist: bool = False):
@@ -388,8 +423,10 @@ class Booster:
             self.phase_marks.append(self._marks)
 
     def step(self, time_hist: bool = False):
-        """One boosting iteration (one tree) on the current stream; asynchronous."""
+        """One boosting iteration (one tree) on the current stream; asynchronous.  With the peer
+        exchange, raises PeerExchangeError as soon as a failed wait of an earlier tree is seen."""
         self._tree(time_hist)
+        self._peer_after_tree()
         if self.keep_model:
             self.trees.append(self.export())
 
@@ -414,6 +451,7 @@ class Booster:
     def fit(self, T: Optional[int] = None):
         for _ in range(T if T is not None else self.params.T):
             self.step()
+        self.check_peer(block=True)
         return self
 
     # ----------------------------------------------------------------- graphs
@@ -421,9 +459,12 @@ class Booster:
         """Capture one tree (grad .. update_pred) as a CUDA graph; replay with step_graph()."""
         s = torch.cuda.Stream(self.device)
         s.wait_stream(torch.cuda.current_stream(self.device))
+        saved = self.pred.clone()             # the warm-up tree is not part of the model
         with torch.cuda.stream(s):
             self._tree()                      # warm-up outside the graph (allocations, attributes)
+            self.pred.copy_(saved)
         torch.cuda.current_stream(self.device).wait_stream(s)
+        del saved
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):
             self._tree()
@@ -432,6 +473,7 @@ class Booster:
 
     def step_graph(self):
         self._graph.replay()
+        self._peer_after_tree()
         if self.keep_model:
             self.trees.append(self.export())
 

@@ -19,7 +19,8 @@ extern "C" gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out) {
   Ctx* ctx = new (std::nothrow) Ctx();
   if (!ctx) return GBDTMO_ENOMEM;
   ctx->device = device;
-  if (cudaSetDevice(device) != cudaSuccess ||
+  DeviceGuard device_guard_(ctx);          // restores the caller's device on return
+  if (cudaGetLastError() != cudaSuccess ||
       cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
       cudaDeviceGetAttribute(&ctx->max_smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device) != cudaSuccess) {
     cudaGetLastError();
@@ -38,6 +39,7 @@ extern "C" gbdtmo_status gbdtmo_destroy(gbdtmo_ctx c) {
 
 extern "C" gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx c, void* stream) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   ctx->stream = (cudaStream_t)stream;
   return GBDTMO_OK;
@@ -45,6 +47,7 @@ extern "C" gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx c, void* stream) {
 
 extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t value) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   switch (option) {
     case GBDTMO_OPT_GMEM_MAX_ROWS: ctx->gmem_max_rows = value; return GBDTMO_OK;
@@ -63,11 +66,13 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
 
 extern "C" const char* gbdtmo_last_error(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   return ctx ? ctx->err.c_str() : "null context";
 }
 
 extern "C" int64_t gbdtmo_launch_count(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   return ctx ? ctx->launches : -1;
 }
 

@@ -505,6 +505,7 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
                                     uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins, void* ws,
                                     size_t ws_bytes) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X && bins && cuts && nbins && ws, "null pointer");
   GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
@@ -514,11 +515,8 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
   GB_CHECK_ARG(B >= 2, "B < 2");
   if (ws_bytes < gbdtmo_bin_workspace_bytes(n, m, B)) { ctx->err = "gbdtmo_bin: workspace too small"; return GBDTMO_ENOMEM; }
   const SelWs w = sel_ws(ws, n, m);
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_bin_apply, cudaFuncAttributeMaxDynamicSharedMemorySize, kBinTC * 255 * 4);
-    attr = true;
-  }
+  static unsigned long long attr_mask = 0;
+  smem_optin_once(ctx, k_bin_apply, attr_mask, kBinTC * 255 * 4);
   for (int c0 = 0; c0 < m; c0 += kBinTC) {
     const int tc = (int)(m - c0 < kBinTC ? m - c0 : kBinTC);
     GB_LAUNCH(k_bin_keys, dim3((unsigned)((n + 31) / 32), (unsigned)((tc + 31) / 32)), dim3(32, 8), 0, X, n, ld_x, c0,
@@ -536,6 +534,7 @@ extern "C" gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx c, const float* values, const
                                         int32_t B, uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                                         void* ws, size_t ws_bytes) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(col_ptr && col_ptr_host && bins && cuts && nbins && ws, "null pointer");
   GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
@@ -571,6 +570,7 @@ extern "C" gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx c, const float* values, const
 extern "C" gbdtmo_status gbdtmo_default_bins(gbdtmo_ctx c, const uint8_t* bins, int64_t n, int32_t m, int64_t ld_bins,
                                              int32_t B, int64_t min_count, int32_t* dflt) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(bins && dflt, "null pointer");
   GB_CHECK_ARG(n >= 1 && m >= 1 && ld_bins >= m && ld_bins % 8 == 0 && B >= 2 && B <= 256, "bad shape");

@@ -31,6 +31,33 @@ struct Ctx {
   std::string err;
 };
 
+// Every entry point runs its CUDA calls on ctx->device and restores the caller's current device
+// on return (the library must not depend on, or change, the caller's current device).
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(const Ctx* ctx) {
+    int cur = -1;
+    if (ctx && cudaGetDevice(&cur) == cudaSuccess && cur != ctx->device) {
+      prev = cur;
+      cudaSetDevice(ctx->device);
+    }
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) applies per device: one bit per device per
+// kernel instantiation (the caller keeps a static mask), set with the context's device current.
+template <typename F>
+inline void smem_optin_once(const Ctx* ctx, F* kernel, unsigned long long& mask, int bytes) {
+  const unsigned long long bit = 1ull << (ctx->device & 63);
+  if (!(__atomic_load_n(&mask, __ATOMIC_ACQUIRE) & bit)) {
+    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    __atomic_fetch_or(&mask, bit, __ATOMIC_RELEASE);
+  }
+}
+
 #define GB_CHECK_ARG(cond, msg)                  \
   do {                                           \
     if (!(cond)) {                               \

@@ -419,12 +419,8 @@ template <int K, int KF, bool SKIP, bool PACKED>
 static gbdtmo_status launch_hist_kfs(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
                                      const uint8_t* packed, const int32_t* dflt, const int32_t* q,
                                      const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_smem<K, KF, SKIP, PACKED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         ctx->max_smem_optin - 1024);
-    attr_done = true;
-  }
+  static unsigned long long attr_mask = 0;
+  smem_optin_once(ctx, k_hist_smem<K, KF, SKIP, PACKED>, attr_mask, ctx->max_smem_optin - 1024);
   GB_LAUNCH((k_hist_smem<K, KF, SKIP, PACKED>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, packed, dflt, q,
             rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
@@ -520,6 +516,7 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
                                            const uint8_t* bins, const int32_t* dflt, const int32_t* q, void* state,
                                            int64_t* hist, int32_t* cnt) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -533,6 +530,7 @@ extern "C" gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx c, const gbdtmo_pro
                                                   const uint8_t* bins, const uint8_t* packed, const int32_t* dflt,
                                                   const int32_t* q, void* state, int64_t* hist, int32_t* cnt) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -552,6 +550,7 @@ extern "C" size_t gbdtmo_packed_bins_bytes(const gbdtmo_problem* p) {
 extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p, const uint8_t* bins,
                                           uint8_t* packed) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -565,6 +564,7 @@ extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p,
 
 extern "C" gbdtmo_status gbdtmo_set_root_counts(gbdtmo_ctx c, const int32_t* root_cnt) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   ctx->root_cnt = root_cnt;
   return GBDTMO_OK;

@@ -229,11 +229,8 @@ template <int KF>
 static gbdtmo_status launch_diag_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const uint8_t* bins,
                                     const int32_t* q, const int32_t* rows, int use_rows, const State& s, int64_t* hist,
                                     int32_t* cnt) {
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_diag<KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin - 1024);
-    attr_done = true;
-  }
+  static unsigned long long attr_mask = 0;
+  smem_optin_once(ctx, k_hist_diag<KF>, attr_mask, ctx->max_smem_optin - 1024);
   GB_LAUNCH(k_hist_diag<KF>, ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
 }

@@ -306,11 +306,8 @@ template <int KF>
 static gbdtmo_status launch_tma_kf(Ctx* ctx, const gbdtmo_problem& p, const HistCfg& hc, const CUtensorMap& tm,
                                    const int32_t* q, const int32_t* rows, int use_rows, const State& s, int64_t* hist,
                                    int32_t* cnt) {
-  static bool attr_done = false;
-  if (!attr_done) {
-    cudaFuncSetAttribute(k_hist_tma<KF>, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin - 1024);
-    attr_done = true;
-  }
+  static unsigned long long attr_mask = 0;
+  smem_optin_once(ctx, k_hist_tma<KF>, attr_mask, ctx->max_smem_optin - 1024);
   GB_LAUNCH(k_hist_tma<KF>, ctx->num_sms, kTmaThreads, hc.smem, p, hc, tm, q, rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
 }

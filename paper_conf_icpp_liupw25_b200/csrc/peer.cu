@@ -109,6 +109,7 @@ extern "C" size_t gbdtmo_peer_window_bytes(const gbdtmo_problem* p) {
 extern "C" gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t rank, int32_t world,
                                           uint8_t* handle) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -122,7 +123,6 @@ extern "C" gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx c, const gbdtmo_problem* p,
   pr->world = world;
   pr->shape = *p;
   pr->bytes = (size_t)peer_window_bytes(*p);
-  cudaSetDevice(ctx->device);
   cudaIpcMemHandle_t h;
   if (cudaMalloc(&pr->own, pr->bytes) != cudaSuccess || cudaMemset(pr->own, 0, pr->bytes) != cudaSuccess ||
       cudaDeviceSynchronize() != cudaSuccess || cudaIpcGetMemHandle(&h, pr->own) != cudaSuccess) {
@@ -140,12 +140,12 @@ extern "C" gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx c, const gbdtmo_problem* p,
 
 extern "C" gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx c, const uint8_t* handles) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(ctx->peer, "gbdtmo_peer_open first");
   GB_CHECK_ARG(handles, "null handles");
   Peer* pr = ctx->peer;
   GB_CHECK_ARG(!pr->connected, "already connected");
-  cudaSetDevice(ctx->device);
   for (int r = 0; r < pr->world; ++r) {
     if (r == pr->rank) continue;
     cudaIpcMemHandle_t h;
@@ -167,6 +167,7 @@ extern "C" gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx c, const uint8_t* handle
 extern "C" gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, uint64_t** keys,
                                              int64_t** xchg) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -179,10 +180,10 @@ extern "C" gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx c, const gbdtmo_problem*
 
 extern "C" gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx c, int64_t* epoch, int64_t* error) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(ctx->peer, "no peer window");
   uint64_t hdr[PEER_HEADER_WORDS];
-  cudaSetDevice(ctx->device);
   if (cudaMemcpy(hdr, ctx->peer->own, sizeof(hdr), cudaMemcpyDeviceToHost) != cudaSuccess) {
     ctx->err = std::string("gbdtmo_peer_status: ") + cudaGetErrorString(cudaGetLastError());
     return GBDTMO_ECUDA;
@@ -192,8 +193,24 @@ extern "C" gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx c, int64_t* epoch, int64_
   return GBDTMO_OK;
 }
 
+extern "C" gbdtmo_status gbdtmo_peer_status_async(gbdtmo_ctx c, int64_t* out) {
+  Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
+  if (!ctx) return GBDTMO_EINVAL;
+  GB_CHECK_ARG(ctx->peer, "no peer window");
+  GB_CHECK_ARG(out, "null output");
+  const uint64_t* hdr = reinterpret_cast<const uint64_t*>(ctx->peer->own);
+  if (cudaMemcpyAsync(out, hdr + PEER_EPOCH, 8, cudaMemcpyDefault, ctx->stream) != cudaSuccess ||
+      cudaMemcpyAsync(out + 1, hdr + PEER_ERROR, 8, cudaMemcpyDefault, ctx->stream) != cudaSuccess) {
+    ctx->err = std::string("gbdtmo_peer_status_async: ") + cudaGetErrorString(cudaGetLastError());
+    return GBDTMO_ECUDA;
+  }
+  return GBDTMO_OK;
+}
+
 extern "C" gbdtmo_status gbdtmo_peer_close(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   peer_release(ctx);
   return GBDTMO_OK;

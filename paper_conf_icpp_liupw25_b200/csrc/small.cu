@@ -234,6 +234,7 @@ extern "C" gbdtmo_status gbdtmo_search_small(gbdtmo_ctx c, const gbdtmo_problem*
                                              const uint8_t* bins, const int32_t* q, const int32_t* nbins,
                                              const float* scales, void* state, uint64_t* keys) {
   Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -253,12 +254,8 @@ extern "C" gbdtmo_status gbdtmo_search_small(gbdtmo_ctx c, const gbdtmo_problem*
   if (fb > fb_max) fb = fb_max;
   if (fb < 1) fb = 1;
   auto kern = p->loss == GBDTMO_LOSS_SOFTMAX ? k_sort_search<true> : k_sort_search<false>;
-  static bool attr_done[2] = {false, false};
-  const int si = p->loss == GBDTMO_LOSS_SOFTMAX;
-  if (!attr_done[si]) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, ctx->max_smem_optin - 1024);
-    attr_done[si] = true;
-  }
+  static unsigned long long attr_mask[2] = {0, 0};
+  smem_optin_once(ctx, kern, attr_mask[p->loss == GBDTMO_LOSS_SOFTMAX], ctx->max_smem_optin - 1024);
   GB_LAUNCH(kern, dim3((unsigned)fb, (unsigned)LN), kSortWarps * 32, L.bytes, *p, level, (int)rcap, bins, q, rows,
             use_rows, nbins, scales, s, keys);
   return GBDTMO_OK;

@@ -394,9 +394,8 @@ def test_graph_replay_equals_eager(pkg, ctx):
     a = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), torch.from_numpy(Y).to(DEV), P)
     a.fit()
     b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), torch.from_numpy(Y).to(DEV), P)
-    b.capture()          # captures (and its warm-up runs) one tree
-    b.pred.zero_()
-    b.trees.clear()
+    b.capture()          # captures one tree; its warm-up tree runs outside the graph and is not kept
+    assert not b.trees and not bool(b.pred.any())       # (the warm-up leaves pred untouched)
     for _ in range(3):
         b.step_graph()
     torch.cuda.synchronize()

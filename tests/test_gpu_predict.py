@@ -8,27 +8,6 @@ from gen import gen
 pytestmark = pytest.mark.gpu
 
 
-def _host_predict(X, cuts, trees, D, d):
-    """Reference walk (test harness): x < cuts[f][b] goes left (reading R15)."""
-    n = X.shape[0]
-    NH = (1 << (D + 1)) - 1
-    out = np.zeros((n, d))
-    for t in range(trees["state"].shape[0]):
-        st, ft, bt, lv = trees["state"][t], trees["feat"][t], trees["bin"][t], trees["leaf"][t]
-        h = np.zeros(n, np.int64)
-        for _ in range(D + 1):
-            s = st[h] == 1
-            if not s.any():
-                break
-            f, b = ft[h[s]], bt[h[s]]
-            go_left = X[np.nonzero(s)[0], f] < cuts[f, b]
-            h[s] = np.where(go_left, 2 * h[s] + 1, 2 * h[s] + 2)
-        assert np.all(st[h] == 2)
-        out += lv[h]
-        assert h.max() < NH
-    return out
-
-
 @pytest.mark.parametrize("case", ["C1", "C3s", "C2s"])
 def test_predict_train_rows_equals_training_prediction_and_oracle_on_unseen(orc, case):
     import paper_conf_icpp_liupw25_b200 as pkg
@@ -50,8 +29,7 @@ def test_predict_train_rows_equals_training_prediction_and_oracle_on_unseen(orc,
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
     ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
                     lr=w.lr, min_node=w.min_node)
-    hu = _host_predict(Xu, cuts, dict(state=ref["state"], feat=ref["feat"], bin=ref["bin"], leaf=ref["leaf"]),
-                       w.D, w.d)
+    hu = orc.predict(Xu, cuts, nbins, w.B, ref, w.D)                 # oracle walk
     assert np.max(np.abs(pu - hu)) <= 1e-4
     # and the exported thresholds are the oracle's cut values
     for t in range(w.T):

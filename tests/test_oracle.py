@@ -379,3 +379,154 @@ def test_train_softmax_invariants(orc):
         z = p - p.max(1, keepdims=True)
         return -np.mean(np.sum(y * (z - np.log(np.exp(z).sum(1, keepdims=True))), 1))
     assert ce(res["pred"]) < ce(p0)
+
+
+# ------------------------------------------------ tie-break (R16) and the split rule gamma (R2, R3)
+
+def _gap_column_problem(n_per=30):
+    """Column 0: integers 0..39 (n_per rows each), rows with x in 15..24 removed from the node, so
+    bins 15..24 are EMPTY in the node; targets depend on x >= 20.  Column 1: noise.  Column 2: an
+    exact copy of column 0 (same bins, same gains at every candidate)."""
+    rng = np.random.default_rng(21)
+    x = np.repeat(np.arange(40), n_per).astype(np.float32)
+    X = np.stack([x, rng.normal(size=len(x)).astype(np.float32), x], 1)
+    y = np.where(x >= 20, 1.0, -1.0)[:, None] + 0.01 * rng.normal(size=(len(x), 1))
+    rows = np.nonzero((x < 15) | (x > 24))[0].astype(np.int32)
+    return X, y, rows
+
+
+def test_tie_break_smallest_feature_then_smallest_bin(orc):
+    """R16: max gain, then smallest feature, then smallest bin.  The best partition of the node
+    ({x <= 14} vs {x >= 25}) is produced by candidates b = 14..24 of column 0 (bins 15..24 are
+    empty in the node: bit-identical gains) and by the same 11 candidates of its copy, column 2.
+    The rule must pick (0, 14); a '>=' slip in the scan picks (2, 24), a feature-only slip (0, 24)."""
+    X, y, rows = _gap_column_problem()
+    cuts, nbins, bins = orc.bin_matrix(X, 64)
+    assert nbins[0] == 40 and nbins[2] == 40
+    g, h = orc.grad(0, y, np.zeros_like(y))
+    HG, HH, CNT = orc.build_hist(bins, 64, g, h, rows)
+    assert np.all(CNT[0][15:25] == 0)
+    sp = orc.find_split(HG, HH, CNT, nbins, g[rows].sum(0), h[rows].sum(0), len(rows), 1.0, 5, want_all=True)
+    allg = sp["all_gains"]
+    assert len(set(allg[0, 14:25].tolist())) == 1 and np.array_equal(allg[0], allg[2])   # the 22-way tie
+    assert np.max(allg[np.isfinite(allg)]) == allg[0, 14]                              # it is the maximum
+    assert (sp["feature"], sp["bin"]) == (0, 14)
+    # independent check of the tie's partition: raw-threshold enumeration (no histograms)
+    gain, f, v = _exhaustive_best(X, g, h, rows, 1.0, 5)
+    assert f == 0 and v == 25.0 and abs(gain - sp["gain"]) <= 1e-7 * abs(gain)
+
+
+def test_tie_break_in_whole_model_prefers_lower_duplicate(orc):
+    """R16 through Algorithm 1: with columns 3 and 7 exact copies of columns 0 and 2, no split of
+    any tree may use column 3 or 7 (each of their candidates ties with the copy's lower index)."""
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    y = gen.targets_host(w, X).astype(np.float64)
+    X = X.copy()
+    X[:, 3] = X[:, 0]
+    X[:, 7] = X[:, 2]
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    res = orc.train(bins, nbins, w.B, y, loss=0, T=5, D=4, lam=1.0, gamma=0.0, lr=1.0, min_node=20)
+    used = res["feat"][res["state"] == 1]
+    assert np.any(np.isin(used, [0, 2]))           # the informative originals are used ...
+    assert not np.any(np.isin(used, [3, 7]))       # ... never their later copies
+
+
+def test_gamma_split_rule_strict(orc):
+    """R2/R3 (Alg. 1 lines 14-17, gamma = 'threshold for valid splits',
+    PAPER.md:122): a node splits iff its best gain > gamma.  gamma = the root's best gain exactly
+    -> the root is a leaf; gamma one ulp below -> it splits."""
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    y = gen.targets_host(w, X).astype(np.float64)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    r0 = orc.train(bins, nbins, w.B, y, T=1, D=3, gamma=0.0)
+    best = r0["gain"][0][0]
+    assert r0["state"][0][0] == 1 and best > 0
+    r_eq = orc.train(bins, nbins, w.B, y, T=1, D=3, gamma=best)
+    assert r_eq["state"][0][0] == 2 and np.all(r_eq["state"][0][1:] == 0)
+    r_lo = orc.train(bins, nbins, w.B, y, T=1, D=3, gamma=np.nextafter(best, 0.0))
+    assert r_lo["state"][0][0] == 1
+
+
+def test_gamma_infinite_gives_root_leaves_closed_form(orc):
+    """gamma larger than any gain: every tree is one root leaf, so for MSE (g = 2(yhat - y), h = 2)
+    yhat_{t+1} = yhat_t - lr * 2 sum(yhat_t - y) / (2 n + lambda) for every row:
+    a closed-form recursion computed here in numpy."""
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    y = gen.targets_host(w, X).astype(np.float64) + 0.75          # off-centre, so leaves are non-zero
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    lam, lr, T = 3.0, 0.4, 4
+    res = orc.train(bins, nbins, w.B, y, T=T, D=4, lam=lam, lr=lr, gamma=1e300)
+    c = np.zeros(w.d)
+    for t in range(T):
+        assert res["state"][t][0] == 2 and np.all(res["state"][t][1:] == 0)
+        c = c - lr * 2.0 * (w.n * c - y.sum(0)) / (2.0 * w.n + lam)
+    np.testing.assert_allclose(res["pred"], np.broadcast_to(c, y.shape), rtol=1e-12, atol=1e-14)
+
+
+@pytest.mark.parametrize("frac", [0.05, 0.1, 0.3])
+def test_gamma_every_node_by_exhaustive_enumeration(orc, frac):
+    """gamma > 0 against raw-threshold enumeration (no histograms): every split node's gain exceeds
+    gamma, and every leaf that could have split (depth < D, >= 2 min_node rows) has no raw
+    threshold with gain > gamma (up to 1e-9 relative)."""
+    X, bins, nbins, y, p = _tiny(31, n=240, m=3, d=2, B=256, loss=0)
+    y = y + 0.2 * X[:, :1].astype(np.float64)
+    g0, h0 = orc.grad(0, y, np.zeros_like(y))
+    root_best = _exhaustive_best(X, g0, h0, np.arange(len(X), dtype=np.int32), 1.0, 10)[0]
+    gamma, D, mn = frac * root_best, 4, 10
+    res = orc.train(bins, nbins, 256, y, T=1, D=D, lam=1.0, gamma=gamma, min_node=mn)
+    from tests.gpu_helpers import node_rows
+    rows = node_rows(bins, res["state"][0], res["feat"][0], res["bin"][0], len(X))
+    n_leaf_checked = 0
+    for hid, r in rows.items():
+        st = res["state"][0][hid]
+        depth = int(np.floor(np.log2(hid + 1)))
+        if st == 1:
+            assert res["gain"][0][hid] > gamma
+        elif st == 2 and depth < D and len(r) >= 2 * mn:
+            best = _exhaustive_best(X, g0, h0, r.astype(np.int32), 1.0, mn)
+            assert best is None or best[0] <= gamma * (1 + 1e-9)
+            n_leaf_checked += 1
+    assert n_leaf_checked > 0 and np.any(res["state"][0] == 1)
+
+
+# ------------------------------------------------------------------ inference (PAPER.md:245)
+
+def test_predict_walk_equals_incremental_training_prediction(orc):
+    """oracle_predict walks every tree from the root on RAW feature values; on the training rows it
+    must reproduce oracle_train's prediction, which never walks a tree (rows carry their leaf,
+    PAPER.md:164) -- two different computations of the same model output."""
+    for w, loss in ((gen.WORKLOADS["C1"].scaled(T=6), 0), (gen.WORKLOADS["C2"].scaled(n=3000, m=30, T=3, D=4), 1)):
+        X = gen.features_host(w)
+        y = gen.targets_host(w, X).astype(np.float64)
+        cuts, nbins, bins = orc.bin_matrix(X, w.B)
+        res = orc.train(bins, nbins, w.B, y, loss=loss, T=w.T, D=w.D, lr=0.7)
+        p = orc.predict(X, cuts, nbins, w.B, res, w.D)
+        np.testing.assert_allclose(p, res["pred"], rtol=0, atol=1e-12)
+
+
+def test_predict_unseen_rows_equals_sklearn_tree_predict(orc):
+    """MSE, lambda = 0, lr = 1: each oracle tree is a CART regressor on the bin matrix (pinned above);
+    on UNSEEN rows the oracle walk over raw values must equal sklearn's tree.predict on the rows'
+    bins (bin(x) from searchsorted on the training cuts)."""
+    from sklearn.tree import DecisionTreeRegressor
+    w = gen.WORKLOADS["C1"]
+    X = gen.features_host(w)
+    y = gen.targets_host(w, X).astype(np.float64)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    T, D = 4, 4
+    res = orc.train(bins, nbins, w.B, y, loss=0, T=T, D=D, lam=0.0, lr=1.0, min_node=20)
+    Xu = gen.features_host(gen.WORKLOADS["C1"].scaled(n=5000), r0=2000, nr=3000)      # rows never trained on
+    Xu = Xu * 1.3 + 0.1                                                               # incl. out-of-range values
+    Bu = np.stack([np.searchsorted(cuts[f][: nbins[f] - 1], Xu[:, f], side="right") for f in range(w.m)], 1)
+    Xb = bins.T.astype(np.float64)
+    pred_tr = np.zeros_like(y)
+    pred_u = np.zeros((len(Xu), w.d))
+    for t in range(T):
+        tree = DecisionTreeRegressor(max_depth=D, min_samples_leaf=20, random_state=0).fit(Xb, y - pred_tr)
+        pred_tr += tree.predict(Xb)
+        pred_u += tree.predict(Bu.astype(np.float64))
+    p = orc.predict(Xu, cuts, nbins, w.B, res, D)
+    np.testing.assert_allclose(p, pred_u, rtol=0, atol=1e-9)

@@ -7,7 +7,7 @@ SRCS    := $(wildcard $(PKG)/csrc/*.cu)
 HDRS    := $(wildcard $(PKG)/csrc/*.cuh) include/gbdtmo.h
 OBJS    := $(patsubst $(PKG)/csrc/%.cu,build/%.o,$(SRCS))
 
-all: $(PKG)/libgbdtmo.so oracle/liboracle.so gen/libgbdtgen.so gen/libgbdtgen_cuda.so
+all: $(PKG)/libgbdtmo.so oracle/liboracle.so gen/libgbdtgen.so gen/libgbdtgen_cuda.so tools/microbench/libgbdtmo_peaks.so
 
 build/%.o: $(PKG)/csrc/%.cu $(HDRS)
 	@mkdir -p build
@@ -25,7 +25,11 @@ gen/libgbdtgen.so: gen/gen.c gen/gen_rng.h
 gen/libgbdtgen_cuda.so: gen/gen_cuda.cu gen/gen_rng.h
 	$(NVCC) $(ARCH) -O3 -lineinfo -Xcompiler -fPIC -shared -o $@ gen/gen_cuda.cu
 
+# same-run roofline denominators for bench.py (measurement only, not the product path)
+tools/microbench/libgbdtmo_peaks.so: tools/microbench/peaks.cu
+	$(NVCC) $(ARCH) -O3 -lineinfo -Xcompiler -fPIC -shared -o $@ $<
+
 clean:
-	rm -rf build $(PKG)/libgbdtmo.so oracle/liboracle.so gen/libgbdtgen.so gen/libgbdtgen_cuda.so
+	rm -rf build $(PKG)/libgbdtmo.so oracle/liboracle.so gen/libgbdtgen.so gen/libgbdtgen_cuda.so tools/microbench/libgbdtmo_peaks.so
 
 .PHONY: all clean

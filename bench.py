@@ -52,6 +52,10 @@ def parse():
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N > 1 (gloo: lets N ranks share one GPU for testing)")
     ap.add_argument("--no-root-cache", action="store_true", help="(A/B) accumulate the root counts every tree")
+    ap.add_argument("--predict", action="store_true",
+                    help="NEXT-3 line: inference throughput (rows x trees / s) of gbdtmo_predict on unseen rows of "
+                         "the workload, with a model of --predict-trees trees trained first (1 GPU)")
+    ap.add_argument("--predict-trees", type=int, default=100)
     ap.add_argument("--exchange", default="auto", choices=["auto", "peer", "collective"],
                     help="N > 1 split exchange: peer = fused peer-memory exchange inside the kernels (NEXT-4), "
                          "collective = torch.distributed all-reduces; auto = peer, verified after the warm-up "
@@ -111,6 +115,28 @@ class ClockSampler:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
         return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(smax), "reasons": sorted(reasons),
                 "samples": len(sm), "power_w_max": max(power)}
+
+
+# ------------------------------------------------------------- same-run roofline denominators
+
+def measure_atoms_peak(device):
+    """Shared-memory atomic ceiling measured in this process right before the timed region
+    (tools/microbench/peaks.cu): mode 0 = conflict-free red.shared.add.u32 (the pipe ceiling, the
+    roofline peak), mode 1 = the histogram kernel's own row-pair lane map.  None if unavailable."""
+    import ctypes as C
+    path = os.path.join(ROOT, "tools", "microbench", "libgbdtmo_peaks.so")
+    if not os.path.exists(path):
+        return None
+    L = C.CDLL(path)
+    L.peaks_atoms.argtypes = [C.c_int, C.c_int, C.c_int] + [C.POINTER(C.c_double)] * 3
+    out = {}
+    for mode, name in ((0, "pipe"), (1, "hist_lane_map")):
+        a, b, c = C.c_double(), C.c_double(), C.c_double()
+        rc = L.peaks_atoms(device, mode, 80_000, C.byref(a), C.byref(b), C.byref(c))
+        if rc != 0:
+            return None
+        out[name] = {"lane_ops_per_clk_sm": a.value, "lane_ops_per_s": b.value, "clk_mhz": c.value}
+    return out
 
 
 # ---------------------------------------------------------------------------- setup
@@ -231,6 +257,11 @@ def main():
     import torch.distributed as dist
     import paper_conf_icpp_liupw25_b200 as pkg
 
+    if a.predict:
+        if rank != 0:
+            return 0
+        return predict_main(a, w, local % torch.cuda.device_count())
+
     local = local % torch.cuda.device_count()       # (ranks may share a GPU with --backend gloo)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -310,6 +341,8 @@ def main():
     if group is not None:
         dist.barrier()
     booster.hist_events.clear()
+    atoms_peak = measure_atoms_peak(local)
+    torch.cuda.synchronize()
 
     # ---- timed region: K trees, device time, max over ranks
     clk = ClockSampler(local)
@@ -337,6 +370,7 @@ def main():
         dist.barrier()
     l1 = ctx.gbdtmo_launch_count()
     clocks = clk.stop()
+    booster.check_peer(block=True)        # a failed peer wait inside the timed region invalidates the run
     ms = e0.elapsed_time(e1)
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if group is not None:
@@ -356,11 +390,24 @@ def main():
     hist_launches = len(hist_ms)
     hist_avg_ms = float(np.sum(hist_ms)) / max(hist_launches, 1)
     V = booster.p.V
-    updates = rows_built * m_loc * (V + 1)               # per built (row, feature): V channels + count
+    by_level = [[built_rows_by_level(tr, w.D)[l] for tr in trees] for l in range(w.D)]
+    rows_lvl = [int(np.sum(v)) for v in by_level]                   # rows built per level, all timed trees
+    root_cached = booster.root_cnt is not None
+    # work per built (row, feature): V channel updates + 1 count (the root's count comes from the cache)
+    updates = sum(r * m_loc * (V + (0 if (l == 0 and root_cached) else 1)) for l, r in enumerate(rows_lvl))
+    lane_ops = sum(r * m_loc * (2 * V + (0 if (l == 0 and root_cached) else 1)) for l, r in enumerate(rows_lvl))
     upd_per_launch = updates / max(hist_launches, 1)
     achieved = upd_per_launch / (hist_avg_ms * 1e-3) if hist_launches else 0.0
-    clock_ghz = 1.965
-    peak = 148 * 16 * clock_ghz * 1e9                     # 32 ATOMS lanes/clk/SM, 2 per update
+    guide_peak_lane = 148 * 32 * 1.965e9                            # 32 ATOMS lanes/clk/SM at the max clock
+    if atoms_peak:
+        peak_lane = atoms_peak["pipe"]["lane_ops_per_s"]
+        peak_src = (f"measured, same run: tools/microbench/peaks.cu red.shared.add.u32 on 32 distinct banks, "
+                    f"{atoms_peak['pipe']['lane_ops_per_clk_sm']:.2f} lane-ops/clk/SM at "
+                    f"{atoms_peak['pipe']['clk_mhz']:.0f} MHz = {atoms_peak['pipe']['lane_ops_per_s'] / 1e12:.2f} "
+                    f"T lane-ops/s; 2 limb atomics per channel update + 1 count per (row, feature)")
+    else:
+        peak_lane, peak_src = guide_peak_lane, "guide (peaks library unavailable): 32 ATOMS lanes/clk/SM x 148 SMs x 1.965 GHz"
+    peak = peak_lane * updates / lane_ops if lane_ops else 0.0      # updates/s at the atomic-pipe ceiling
     alg_bytes = rows_built * (m_loc + 4 * V + 4)          # bins + q + row id per built row
     hbm_gbs = alg_bytes / max(hist_launches, 1) / (hist_avg_ms * 1e-3) / 1e9 if hist_launches else 0.0
     peaks = {}
@@ -370,11 +417,16 @@ def main():
         pass
     hbm_peak = float(peaks.get("hbm_gbs") or 6650.0)      # B200_PROFILING.md fallback when the file is absent
     hbm_peak_src = "MEASURED_PEAKS.json hbm_gbs" if peaks.get("hbm_gbs") else "of fallback (B200_PROFILING.md: 6.65 TB/s)"
-    traffic = None
+    # DRAM traffic: bytes per built row per level from an ncu --set full capture of this bench's own
+    # timed histogram launches (profiles/hist_traffic.json, tools/traffic_capture.sh), applied to the
+    # rows this run built
+    traffic, traffic_src = None, None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "hist_traffic.json")))
-        if prof.get("workload") == w.name and world == 1:     # (captured on one GPU, all features)
-            traffic = prof.get("dram_bytes_per_launch")
+        bpr = prof.get("dram_bytes_per_built_row_by_level")
+        if prof.get("workload") == w.name and world == 1 and bpr and len(bpr) == w.D:
+            traffic = sum(b * r for b, r in zip(bpr, rows_lvl)) / max(hist_launches, 1)
+            traffic_src = prof.get("source")
     except (OSError, ValueError):
         pass
 
@@ -400,11 +452,20 @@ def main():
         "roofline": {"bound": "alu", "kernel": "k_hist_smem (+k_zero_build) via gbdtmo_build_hist",
                      "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tupdate/s",
                      "frac": achieved / peak if peak else None, "traffic": traffic,
-                     "peak_source": "guide: 32 banks x 4 B/clk/SM shared pipe -> 32 int32 ATOMS lanes/clk/SM, "
-                                    "2 limbs per update, 148 SMs, 1.965 GHz max clock (DESIGN.md Roofline)",
+                     "peak_source": peak_src,
+                     "frac_of_guide_peak": (achieved / (guide_peak_lane * updates / lane_ops)) if lane_ops else None,
+                     "hbm_frac": hbm_gbs / hbm_peak,
                      "hbm_view": {"achieved_gbs": hbm_gbs, "peak_gbs": hbm_peak, "frac": hbm_gbs / hbm_peak,
-                                  "peak_source": hbm_peak_src},
+                                  "peak_source": hbm_peak_src,
+                                  "bytes": "algorithmic per built row: m bins + 4V q + 4 row id (north star's definition)"},
+                     "traffic_source": traffic_src, "traffic_per_built_row": traffic * hist_launches / rows_built
+                     if traffic else None,
+                     "atoms_microbench": atoms_peak,
                      "launches": hist_launches, "avg_launch_ms": hist_avg_ms},
+        "work": {"rows_built_per_tree": rows_built / a.steps, "logical_rows_per_tree": ro / w.d / a.steps,
+                 "hist_ns_per_built_row": hist_total_ms * 1e6 / max(rows_built, 1),
+                 "ms_per_tree_per_M_rows_built": ms_per_tree / (rows_built / a.steps / 1e6) if rows_built else None,
+                 "note": "trees differ in rows built (which children are smaller); compare runs per built row"},
         "clocks": clocks,
         "gpu_launches": int(l1 - l0),
     }
@@ -428,6 +489,80 @@ def main():
         print(json.dumps(out))
     if group is not None:
         dist.destroy_process_group()
+    return 0
+
+
+def predict_main(a, w, local):
+    """Inference line: train a model of --predict-trees trees on the
+    workload, then time K passes of gbdtmo_predict over n UNSEEN rows (rows n..2n-1 of the same
+    generator) resident in HBM.  value = rows x trees / s.  The kernel stages every row (m floats)
+    once per pass, so it is bound by reading X from HBM: roofline bound "hbm", bytes = n m 4."""
+    import torch
+    import paper_conf_icpp_liupw25_b200 as pkg
+    from gen import gen
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    ctx = pkg.Context(local)
+    T = a.predict_trees
+
+    def device_X(r0):
+        if w.classes_sweep:
+            return torch.from_numpy(gen.features_host(w, r0, w.n)).to(dev)
+        X = torch.empty((w.n, w.m), dtype=torch.float32, device=dev)
+        gen.matrix_cuda(w.seed, gen.STREAM_X, w.x_kind, r0, w.n, 0, w.m, w.m, X.data_ptr(), w.m,
+                        torch.cuda.current_stream().cuda_stream)
+        return X
+    X = device_X(0)
+    ds = pkg.bin_features(ctx, X, w.B)
+    del X
+    torch.cuda.empty_cache()
+    Y = torch.from_numpy(host_targets(w)).to(dev)
+    params = pkg.Params(loss=w.loss, T=T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+    b = pkg.Booster(ctx, ds, Y, params)
+    t0 = time.perf_counter()
+    b.fit()
+    torch.cuda.synchronize()
+    train_s = time.perf_counter() - t0
+    trees = b.trees
+    del b, ds, Y
+    torch.cuda.empty_cache()
+    Xu = device_X(w.n)                                   # unseen rows
+    pred = torch.zeros((w.n, w.d), dtype=torch.float64, device=dev)
+    for _ in range(a.warmup):
+        pkg.predict(ctx, trees, Xu, w.D, w.d, pred=pred)
+    torch.cuda.synchronize()
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    l0 = ctx.gbdtmo_launch_count()
+    e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(a.steps):
+        pkg.predict(ctx, trees, Xu, w.D, w.d, pred=pred)
+    e1.record()
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1) / a.steps
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except OSError:
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs") or 6650.0)
+    xbytes = w.n * w.m * 4
+    gbs = xbytes / (ms * 1e-3) / 1e9
+    out = {"metric": "inference rows*trees/s (gbdtmo_predict, unseen rows)", "value": w.n * T / (ms * 1e-3),
+           "unit": "rows*trees/s", "n_gpus": 1, "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32 compare, f64 sums",
+           "data": "synthetic (seeded counter-based generator, gen/); unseen rows n..2n-1, in HBM",
+           "config": {"workload": w.name, "n": w.n, "m": w.m, "d": w.d, "D": w.D, "trees": T,
+                      "l2": "inputs larger than L2" if xbytes > 126e6 else "X fits L2"},
+           "train_s_for_model": train_s,
+           "roofline": {"bound": "hbm", "kernel": "k_predict_tiles", "achieved": gbs, "peak": hbm_peak,
+                        "unit": "GB/s", "frac": gbs / hbm_peak, "traffic": None,
+                        "bytes": "n x m x 4 (every row staged once per pass)"},
+           "clocks": clocks, "gpu_launches": int(ctx.gbdtmo_launch_count() - l0)}
+    print(json.dumps(out))
     return 0
 
 

@@ -89,7 +89,7 @@ def lib():
             "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
-            "gbdtmo_predict": ([P, P, i64, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
+            "gbdtmo_predict": ([P, P, i64, i32, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
             "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
             "gbdtmo_set_root_counts": ([P, P], C.c_int),
             "gbdtmo_peer_window_bytes": ([PP], sz),
@@ -255,8 +255,8 @@ class Context:
                                              _ptr(bin), _ptr(gain), _ptr(n_rows), _ptr(n_left), _ptr(cuts),
                                              _ptr(threshold)), "gbdtmo_tree_export")
 
-    def gbdtmo_predict(self, X, n, ld_x, T, D, d, node_state, feature, threshold, leaf, pred):
-        self._check(lib().gbdtmo_predict(self._h, _ptr(X), n, ld_x, T, D, d, _ptr(node_state), _ptr(feature),
+    def gbdtmo_predict(self, X, n, m, ld_x, T, D, d, node_state, feature, threshold, leaf, pred):
+        self._check(lib().gbdtmo_predict(self._h, _ptr(X), n, m, ld_x, T, D, d, _ptr(node_state), _ptr(feature),
                                          _ptr(threshold), _ptr(leaf), _ptr(pred)), "gbdtmo_predict")
 
     def gbdtmo_rows_export(self, p, state, level, rows=None, node_of_row=None, node_begin=None, node_end=None):

@@ -515,5 +515,5 @@ def predict(ctx: Context, trees, X: torch.Tensor, D: int, d: int, pred: Optional
     th = torch.stack([t["threshold"] for t in trees]).contiguous()
     lf = torch.stack([t["leaf"] for t in trees]).contiguous()
     ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
-    ctx.gbdtmo_predict(X, n, X.stride(0), T, D, d, st, ft, th, lf, pred)
+    ctx.gbdtmo_predict(X, n, X.shape[1], X.stride(0), T, D, d, st, ft, th, lf, pred)
     return pred

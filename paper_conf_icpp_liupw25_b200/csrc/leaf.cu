@@ -59,27 +59,74 @@ __global__ void k_tree_export(gbdtmo_problem p, State s, int32_t* node_state, in
 
 // One warp per instance: all lanes walk the (uniform) path of each tree, lanes add the leaf's
 // outputs (coalesced); trees in order so the sums match the training-time accumulation.
-__global__ void k_predict(const float* __restrict__ X, int64_t n, int64_t ld_x, int T, int D, int d,
-                          const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
-                          const float* __restrict__ threshold, const double* __restrict__ leaf,
-                          double* __restrict__ pred) {
-  const int lane = threadIdx.x & 31;
+// Inference for unseen rows (instance-level and tree-level parallelism).
+// A block owns a tile of RB rows at a time (persistent over tiles):
+//   1. the tile's rows are staged in shared memory (coalesced; row stride mp = m | 1, so 32 rows
+//      reading the same feature hit 32 different banks);
+//   2. tree-level x instance-level walk: thread pairs (row r, tree t) of a chunk of TC trees walk
+//      tree t from the root for row r (x < threshold -> left, reading R15) and park the leaf id
+//      in shared memory; consecutive lanes take consecutive rows of the same tree, so node
+//      loads are broadcast near the root;
+//   3. lanes over (row, output) add the chunk's leaf values in tree order (fp64, the same
+//      sequential order as the training path's update_pred, so predictions of training rows are
+//      bit-identical to the training prediction).
+// Without staging (rows wider than the shared-memory budget) the walk reads X from global memory.
+__global__ void __launch_bounds__(256)
+k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int T, int D, int d, int RB, int TC,
+                int stage, const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
+                const float* __restrict__ threshold, const double* __restrict__ leaf, double* __restrict__ pred) {
+  extern __shared__ __align__(16) unsigned char smp[];
+  const int mp = m | 1;
+  float* xs = reinterpret_cast<float*>(smp);
+  int16_t* lh = reinterpret_cast<int16_t*>(smp + (stage ? (size_t)RB * mp * 4 : 0));
   const int64_t NH = (int64_t(1) << (D + 1)) - 1;
-  const int64_t wpb = blockDim.x >> 5;
-  for (int64_t i = blockIdx.x * wpb + (threadIdx.x >> 5); i < n; i += (int64_t)gridDim.x * wpb) {
-    const float* xi = X + i * ld_x;
-    double* pi = pred + i * d;
-    for (int t = 0; t < T; ++t) {
-      const int32_t* st = node_state + (int64_t)t * NH;
-      int64_t h = 0;
-      while (h < NH && st[h] == GBDTMO_NODE_SPLIT) {
-        const int32_t f = feature[(int64_t)t * NH + h];
-        h = (xi[f] < threshold[(int64_t)t * NH + h]) ? 2 * h + 1 : 2 * h + 2;
+  const int64_t ntiles = (n + RB - 1) / RB;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t r0 = tile * RB;
+    const int rows = (int)min((int64_t)RB, n - r0);
+    if (stage) {
+      for (int e = threadIdx.x; e < RB * m; e += blockDim.x) {
+        const int r = e / m, j = e - r * m;
+        xs[r * mp + j] = r < rows ? __ldg(&X[(r0 + r) * ld_x + j]) : 0.f;
       }
-      if (h < NH && st[h] == GBDTMO_NODE_LEAF) {
-        const double* lv = leaf + ((int64_t)t * NH + h) * d;
-        for (int k = lane; k < d; k += 32) pi[k] += lv[k];
+      __syncthreads();
+    }
+    for (int t0 = 0; t0 < T; t0 += TC) {
+      const int tc = min(TC, T - t0);
+      for (int pq = threadIdx.x; pq < RB * tc; pq += blockDim.x) {
+        const int r = pq % RB, t = pq / RB;
+        int h = -1;
+        if (r < rows) {
+          const int32_t* st = node_state + (int64_t)(t0 + t) * NH;
+          const int32_t* ft = feature + (int64_t)(t0 + t) * NH;
+          const float* th = threshold + (int64_t)(t0 + t) * NH;
+          const float* xr = stage ? xs + r * mp : X + (r0 + r) * ld_x;
+          int64_t c = 0;
+          int sc = __ldg(&st[0]);
+          while (sc == GBDTMO_NODE_SPLIT) {
+            const int f = __ldg(&ft[c]);
+            if ((unsigned)f >= (unsigned)m) { sc = GBDTMO_NODE_NONE; break; }   // (malformed model)
+            const float x = stage ? xr[f] : __ldg(&xr[f]);
+            c = (x < __ldg(&th[c])) ? 2 * c + 1 : 2 * c + 2;
+            sc = c < NH ? __ldg(&st[c]) : GBDTMO_NODE_NONE;
+          }
+          h = sc == GBDTMO_NODE_LEAF ? (int)c : -1;
+        }
+        lh[r * TC + t] = (int16_t)h;
       }
+      __syncthreads();
+      for (int e = threadIdx.x; e < rows * d; e += blockDim.x) {
+        const int r = e / d, k = e - r * d;
+        double* pp = pred + (r0 + r) * d + k;
+        double acc = *pp;
+        const int16_t* hr = lh + r * TC;
+        for (int t = 0; t < tc; ++t) {
+          const int h = hr[t];
+          if (h >= 0) acc += __ldg(&leaf[((int64_t)(t0 + t) * NH + h) * d + k]);
+        }
+        *pp = acc;
+      }
+      __syncthreads();
     }
   }
 }
@@ -157,15 +204,31 @@ extern "C" gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx c, const gbdtmo_problem* 
   return GBDTMO_OK;
 }
 
-extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n, int64_t ld_x, int32_t T, int32_t D,
-                                        int32_t d, const int32_t* node_state, const int32_t* feature,
+extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t T,
+                                        int32_t D, int32_t d, const int32_t* node_state, const int32_t* feature,
                                         const float* threshold, const double* leaf, double* pred) {
   Ctx* ctx = (Ctx*)c;
   DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X && node_state && feature && threshold && leaf && pred, "null pointer");
-  GB_CHECK_ARG(n >= 0 && T >= 0 && D >= 0 && D <= 20 && d >= 1, "bad shape");
+  GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");
+  GB_CHECK_ARG(D >= 1 && D <= 12, "D out of range [1, 12]");
   if (n == 0 || T == 0) return GBDTMO_OK;
-  GB_LAUNCH(k_predict, ctx->num_sms * 8, 256, 0, X, n, ld_x, T, D, d, node_state, feature, threshold, leaf, pred);
+  // rows per tile: the largest power of two <= 64 whose staged rows fit 160 KB (0: no staging)
+  const int64_t row_bytes = 4 * (int64_t)(m | 1);
+  int RB = 64;
+  while (RB > 1 && RB * row_bytes > 160 * 1024) RB >>= 1;
+  const int stage = RB * row_bytes <= 160 * 1024;
+  if (!stage) RB = 64;
+  const int TC = T < 256 ? T : 256;
+  const int smem = (stage ? (int)(RB * row_bytes) : 0) + RB * TC * 2;
+  static unsigned long long attr_mask = 0;
+  smem_optin_once(ctx, k_predict_tiles, attr_mask, 200 * 1024);
+  const int64_t ntiles = (n + RB - 1) / RB;
+  const int per_sm = smem > 0 ? (int)((ctx->max_smem_optin) / (smem + 1024)) : 8;
+  int64_t grid = (int64_t)ctx->num_sms * (per_sm < 1 ? 1 : per_sm > 8 ? 8 : per_sm);
+  if (grid > ntiles) grid = ntiles;
+  GB_LAUNCH(k_predict_tiles, (unsigned)grid, 256, smem, X, n, m, ld_x, T, D, d, RB, TC, stage, node_state, feature,
+            threshold, leaf, pred);
   return GBDTMO_OK;
 }

@@ -23,7 +23,7 @@ def test_library_exports_every_declared_symbol():
     for n in names:
         assert hasattr(L, n), n
     assert set(names) == set(_abi.SYMBOLS)
-    assert L.gbdtmo_abi_version() == 1
+    assert L.gbdtmo_abi_version() == 2
 
 
 def test_sizes_and_validation_on_host():

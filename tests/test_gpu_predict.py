@@ -37,3 +37,30 @@ def test_predict_train_rows_equals_training_prediction_and_oracle_on_unseen(orc,
         thr = b.trees[t]["threshold"].cpu().numpy()
         sp = st == 1
         np.testing.assert_array_equal(thr[sp], cuts[ref["feat"][t][sp], ref["bin"][t][sp]])
+
+
+@pytest.mark.parametrize("n,m,T,D", [(3000, 3000, 4, 5),      # 8-row tiles staged in shared memory
+                                     (700, 50_000, 3, 4),      # rows too wide to stage: global reads
+                                     (2500, 12, 300, 2)])      # > 256 trees: tree chunks
+def test_predict_shapes_vs_oracle_walk(orc, n, m, T, D):
+    """gbdtmo_predict on wide rows, unstaged rows and multi-chunk forests: the GPU's exported trees
+    walked by the oracle (oracle_predict) on the GPU trees' own (feature, bin) and
+    the oracle's cuts of the same training columns; training rows reproduce the training pred."""
+    import paper_conf_icpp_liupw25_b200 as pkg
+    w = gen.WORKLOADS["C3"].scaled(n=n, m=m, T=T, D=D)
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    ctx = pkg.Context(0)
+    P = pkg.Params(loss=0, T=T, D=D, B=w.B, lr=0.3, min_node=5)
+    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P)
+    b.fit()
+    pt = pkg.predict(ctx, b.trees, torch.from_numpy(X).cuda(), D, w.d)
+    torch.cuda.synchronize()
+    assert torch.equal(pt, b.pred)
+    Xu = gen.features_host(w, r0=n, nr=1111) * 1.5
+    pu = pkg.predict(ctx, b.trees, torch.from_numpy(Xu).cuda(), D, w.d).cpu().numpy()
+    cuts, nbins, _ = orc.bin_matrix(X, w.B)
+    trees = {k: np.stack([t[kk].cpu().numpy() for t in b.trees]) for k, kk in
+             (("state", "node_state"), ("feat", "feature"), ("bin", "bin"), ("leaf", "leaf"))}
+    ref = orc.predict(Xu, cuts, nbins, w.B, trees, D)
+    np.testing.assert_allclose(pu, ref, rtol=0, atol=1e-12)

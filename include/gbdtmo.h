@@ -135,8 +135,10 @@ size_t gbdtmo_bins_bytes(int64_t n, int64_t ld_bins);
 size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B);
 /* Opaque per-tree state (row lists, per-row node ids, heap node tables, launch plans). */
 gbdtmo_status gbdtmo_state_bytes(const gbdtmo_problem* p, size_t* bytes /* host */);
-/* Histogram buffers of one level: hist int64 [2^level][m][V][B] (channel-major: bins contiguous),
- * cnt int32 [2^level][m][B]. */
+/* Histogram buffers of one level: hist int64 [S][m][V][B] (channel-major: bins contiguous),
+ * cnt int32 [S][m][B], S = 2^level slots, except at the last level (level = D-1 > 0), where only
+ * the built child of each sibling pair is materialised and S = 2^(D-2): node `slot` of that level
+ * lives in slot >> 1. */
 gbdtmo_status gbdtmo_hist_bytes(const gbdtmo_problem* p, int32_t level, size_t* hist_bytes, size_t* cnt_bytes);
 /* Exchange buffer (int64 elements): 2^(D-1) split records of V+4 words, then ceil(n/64) bitmap words. */
 gbdtmo_status gbdtmo_xchg_count(const gbdtmo_problem* p, int64_t* count /* host */);
@@ -204,7 +206,8 @@ gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* 
  * (§3.3; the paper's Alg. 2 body is missing.)
  * bins uint8 with ld = p->ld_bins and gbdtmo_bins_bytes() of storage; q from gbdtmo_grad;
  * hist / cnt: this level's buffers (gbdtmo_hist_bytes(level)); slot = node index within the
- * level (heap id - (2^level - 1)).  Slots not built are left untouched.
+ * level (heap id - (2^level - 1)), stored at slot >> 1 on the last level.  Slots not built are
+ * left untouched.
  * dflt (may be NULL): per-feature default bins (gbdtmo_default_bins); rows in a feature's
  * default bin are not accumulated and that bin's entries are left undefined until
  * gbdtmo_find_split recovers them from the node totals. */

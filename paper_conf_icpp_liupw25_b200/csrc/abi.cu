@@ -87,7 +87,7 @@ extern "C" gbdtmo_status gbdtmo_state_bytes(const gbdtmo_problem* p, size_t* byt
 extern "C" gbdtmo_status gbdtmo_hist_bytes(const gbdtmo_problem* p, int32_t level, size_t* hist_bytes,
                                            size_t* cnt_bytes) {
   if (check_problem(p) || level < 0 || level >= p->D) return GBDTMO_EINVAL;
-  const size_t LN = size_t(1) << level;
+  const size_t LN = (size_t)hist_slots(*p, level);
   if (hist_bytes) *hist_bytes = LN * (size_t)p->m * p->B * channels(*p) * 8;
   if (cnt_bytes) *cnt_bytes = LN * (size_t)p->m * p->B * 4;
   return GBDTMO_OK;

@@ -111,6 +111,17 @@ __host__ __device__ inline int64_t max_chunks(const gbdtmo_problem& p) {
   return p.n / kChunkMin + (int64_t(1) << p.D) + 2;
 }
 __host__ __device__ inline int64_t part_tiles(const gbdtmo_problem& p) { return (p.n + kPartTile - 1) / kPartTile; }
+// Histogram slot of node `slot` (index within its level) in that level's buffer.  At the last
+// level (D-1 > 0) only the BUILT child of each sibling pair is ever materialised (the derived
+// one is searched as parent - built and never written), so the pair shares slot >> 1: the last
+// level's buffer holds 2^(D-2) nodes instead of 2^(D-1) (C5 at D = 11 and a
+// Delicious-shaped d = 983 problem at depth 8 fit in HBM).
+__host__ __device__ inline int64_t hist_index(const gbdtmo_problem& p, int level, int64_t slot) {
+  return (level == p.D - 1 && level > 0) ? (slot >> 1) : slot;
+}
+__host__ __device__ inline int64_t hist_slots(const gbdtmo_problem& p, int level) {
+  return (level == p.D - 1 && level > 0) ? (int64_t(1) << (level - 1)) : (int64_t(1) << level);
+}
 __host__ __device__ inline int64_t rec_words(const gbdtmo_problem& p) { return channels(p) + 4; }
 __host__ __device__ inline int64_t bitmap_offset(const gbdtmo_problem& p) { return max_level_nodes(p) * rec_words(p); }
 

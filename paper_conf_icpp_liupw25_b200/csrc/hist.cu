@@ -403,8 +403,8 @@ __global__ void k_zero_build(gbdtmo_problem p, int level, State s, int64_t* __re
   const int64_t V = channels(p);
   const int64_t hw = (int64_t)p.m * p.B * V;           // int64 words per slot
   const int64_t cw = (int64_t)p.m * p.B;               // int32 words per slot
-  int64_t* hb = hist + slot * hw;
-  int32_t* cb = cnt + slot * cw;
+  int64_t* hb = hist + hist_index(p, level, slot) * hw;
+  int32_t* cb = cnt + hist_index(p, level, slot) * cw;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   // hw is even when V is even; handle generally with a scalar tail
   const int64_t hv = hw / 2;

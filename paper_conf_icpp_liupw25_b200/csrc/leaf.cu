@@ -71,48 +71,56 @@ __global__ void k_tree_export(gbdtmo_problem p, State s, int32_t* node_state, in
 //      sequential order as the training path's update_pred, so predictions of training rows are
 //      bit-identical to the training prediction).
 // Without staging (rows wider than the shared-memory budget) the walk reads X from global memory.
-__global__ void __launch_bounds__(256)
-k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int T, int D, int d, int RB, int TC,
+constexpr int kPredThreads = 512;
+
+__global__ void __launch_bounds__(kPredThreads)
+k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int T, int D, int d, int lrb, int TC,
                 int stage, const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
                 const float* __restrict__ threshold, const double* __restrict__ leaf, double* __restrict__ pred) {
   extern __shared__ __align__(16) unsigned char smp[];
+  const int RB = 1 << lrb;
   const int mp = m | 1;
   float* xs = reinterpret_cast<float*>(smp);
   int16_t* lh = reinterpret_cast<int16_t*>(smp + (stage ? (size_t)RB * mp * 4 : 0));
   const int64_t NH = (int64_t(1) << (D + 1)) - 1;
-  const int64_t ntiles = (n + RB - 1) / RB;
+  const int64_t ntiles = (n + RB - 1) >> lrb;
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-    const int64_t r0 = tile * RB;
+    const int64_t r0 = tile << lrb;
     const int rows = (int)min((int64_t)RB, n - r0);
     if (stage) {
-      for (int e = threadIdx.x; e < RB * m; e += blockDim.x) {
-        const int r = e / m, j = e - r * m;
-        xs[r * mp + j] = r < rows ? __ldg(&X[(r0 + r) * ld_x + j]) : 0.f;
+      for (int r = 0; r < RB; ++r) {
+        const float* src = X + (r0 + r) * ld_x;
+        float* dst = xs + r * mp;
+        if (r < rows) {
+          for (int j = threadIdx.x; j < m; j += blockDim.x) dst[j] = __ldg(&src[j]);
+        }
       }
       __syncthreads();
     }
     for (int t0 = 0; t0 < T; t0 += TC) {
       const int tc = min(TC, T - t0);
-      for (int pq = threadIdx.x; pq < RB * tc; pq += blockDim.x) {
-        const int r = pq % RB, t = pq / RB;
+      for (int pq = threadIdx.x; pq < (tc << lrb); pq += blockDim.x) {
+        const int r = pq & (RB - 1), t = pq >> lrb;
         int h = -1;
         if (r < rows) {
-          const int32_t* st = node_state + (int64_t)(t0 + t) * NH;
-          const int32_t* ft = feature + (int64_t)(t0 + t) * NH;
-          const float* th = threshold + (int64_t)(t0 + t) * NH;
+          const int64_t to = (int64_t)(t0 + t) * NH;
           const float* xr = stage ? xs + r * mp : X + (r0 + r) * ld_x;
           int64_t c = 0;
-          int sc = __ldg(&st[0]);
+          int sc = __ldg(&node_state[to]);
+          int f = __ldg(&feature[to]);
+          float th = __ldg(&threshold[to]);
           while (sc == GBDTMO_NODE_SPLIT) {
-            const int f = __ldg(&ft[c]);
             if ((unsigned)f >= (unsigned)m) { sc = GBDTMO_NODE_NONE; break; }   // (malformed model)
             const float x = stage ? xr[f] : __ldg(&xr[f]);
-            c = (x < __ldg(&th[c])) ? 2 * c + 1 : 2 * c + 2;
-            sc = c < NH ? __ldg(&st[c]) : GBDTMO_NODE_NONE;
+            c = (x < th) ? 2 * c + 1 : 2 * c + 2;
+            if (c >= NH) { sc = GBDTMO_NODE_NONE; break; }
+            sc = __ldg(&node_state[to + c]);            // the three loads of the next node are independent
+            f = __ldg(&feature[to + c]);
+            th = __ldg(&threshold[to + c]);
           }
           h = sc == GBDTMO_NODE_LEAF ? (int)c : -1;
         }
-        lh[r * TC + t] = (int16_t)h;
+        lh[(r * TC) + t] = (int16_t)h;
       }
       __syncthreads();
       for (int e = threadIdx.x; e < rows * d; e += blockDim.x) {
@@ -214,21 +222,24 @@ extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n,
   GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");
   GB_CHECK_ARG(D >= 1 && D <= 12, "D out of range [1, 12]");
   if (n == 0 || T == 0) return GBDTMO_OK;
-  // rows per tile: the largest power of two <= 64 whose staged rows fit 160 KB (0: no staging)
+  // rows per tile: the largest power of two <= 64 whose staged rows fit 72 KB, so 2-3 blocks share an
+  // SM and one block's staging overlaps the others' walks (0: rows too wide, read from global memory)
   const int64_t row_bytes = 4 * (int64_t)(m | 1);
-  int RB = 64;
-  while (RB > 1 && RB * row_bytes > 160 * 1024) RB >>= 1;
-  const int stage = RB * row_bytes <= 160 * 1024;
-  if (!stage) RB = 64;
+  int lrb = 6;
+  while (lrb > 0 && (int64_t(1) << lrb) * row_bytes > 72 * 1024) --lrb;
+  const int stage = (int64_t(1) << lrb) * row_bytes <= 72 * 1024;
+  if (!stage) lrb = 5;
+  const int RB = 1 << lrb;
   const int TC = T < 256 ? T : 256;
   const int smem = (stage ? (int)(RB * row_bytes) : 0) + RB * TC * 2;
   static unsigned long long attr_mask = 0;
   smem_optin_once(ctx, k_predict_tiles, attr_mask, 200 * 1024);
   const int64_t ntiles = (n + RB - 1) / RB;
-  const int per_sm = smem > 0 ? (int)((ctx->max_smem_optin) / (smem + 1024)) : 8;
-  int64_t grid = (int64_t)ctx->num_sms * (per_sm < 1 ? 1 : per_sm > 8 ? 8 : per_sm);
+  int per_sm = (int)(ctx->max_smem_optin / (smem + 1024));
+  per_sm = per_sm < 1 ? 1 : per_sm > 4 ? 4 : per_sm;
+  int64_t grid = (int64_t)ctx->num_sms * per_sm;
   if (grid > ntiles) grid = ntiles;
-  GB_LAUNCH(k_predict_tiles, (unsigned)grid, 256, smem, X, n, m, ld_x, T, D, d, RB, TC, stage, node_state, feature,
-            threshold, leaf, pred);
+  GB_LAUNCH(k_predict_tiles, (unsigned)grid, kPredThreads, smem, X, n, m, ld_x, T, D, d, lrb, TC, stage, node_state,
+            feature, threshold, leaf, pred);
   return GBDTMO_OK;
 }

@@ -77,7 +77,7 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     for (int c = 0; c < nchunk; ++c) {
       int cb = b + c * R;
       int ce = cb + R < e ? cb + R : e;
-      s.chunks[off + c] = make_int4((int)i, cb, ce, nchunk == 1 ? 1 : 0);   // w = 1: sole writer
+      s.chunks[off + c] = make_int4((int)hist_index(p, level, i), cb, ce, nchunk == 1 ? 1 : 0);   // w = 1: sole writer
     }
     if (nchunk == 1) s.node_mode[first + i] = MODE_BUILD1;
     __syncthreads();
@@ -104,7 +104,7 @@ __device__ inline void plan_level_chunks(const gbdtmo_problem& p, const State& s
     int tn, tr;
     const int on = block_excl_scan_256(take, &tn);
     const int orow = block_excl_scan_256(rows, &tr);
-    if (take) s.gnodes[sh_gn + on] = make_int4((int)i, b, e, sh_gr + orow);
+    if (take) s.gnodes[sh_gn + on] = make_int4((int)hist_index(p, level, i), b, e, sh_gr + orow);
     __syncthreads();
     if (threadIdx.x == 0) { sh_gn += tn; sh_gr += tr; }
     __syncthreads();

@@ -136,7 +136,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
     long long cl[kFsBins];
     long long ctot;
     {
-      const int64_t oc = ((int64_t)slot * m + f) * B, os = ((int64_t)sib * m + f) * B, op = ((int64_t)par * m + f) * B;
+      const int64_t oc = (hist_index(p, level, slot) * m + f) * B, os = (hist_index(p, level, sib) * m + f) * B, op = ((int64_t)par * m + f) * B;
 #pragma unroll
       for (int i = 0; i < kFsBins; ++i) {
         const int b = b0 + i;
@@ -152,7 +152,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
       if (own && db >= b0 && db < b0 + kFsBins) cnt[oc + db] = (int32_t)dc;   // recovered default-bin count
     }
     // ---- channels
-    const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
+    const int64_t rowc = (hist_index(p, level, slot) * m + f) * V * B, rows_ = (hist_index(p, level, sib) * m + f) * V * B,
                   rowp = ((int64_t)par * m + f) * V * B;
     double accL[kFsBins], accR[kFsBins];
 #pragma unroll
@@ -350,7 +350,7 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
     long long cl[kFsHBins];
     const long long ctot = S[V];
     {
-      const int64_t oc = ((int64_t)slot * m + f) * B, os = ((int64_t)sib * m + f) * B, op = ((int64_t)par * m + f) * B;
+      const int64_t oc = (hist_index(p, level, slot) * m + f) * B, os = (hist_index(p, level, sib) * m + f) * B, op = ((int64_t)par * m + f) * B;
 #pragma unroll
       for (int i = 0; i < kFsHBins; ++i) {
         const int b = b0 + i;
@@ -367,7 +367,7 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
         for (int i = 0; i < kFsHBins; ++i) cl[i] = ctot - cl[i];
       }
     }
-    const int64_t rowc = ((int64_t)slot * m + f) * V * B, rows_ = ((int64_t)sib * m + f) * V * B,
+    const int64_t rowc = (hist_index(p, level, slot) * m + f) * V * B, rows_ = (hist_index(p, level, sib) * m + f) * V * B,
                   rowp = ((int64_t)par * m + f) * V * B;
     double accL[kFsHBins], accR[kFsHBins];
 #pragma unroll
@@ -531,7 +531,7 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
   }
   const bool derive = s.node_mode[h] == MODE_DERIVE;
   const int sib = slot ^ 1, par = slot >> 1;
-  const int64_t rc = ((int64_t)slot * m + fl) * B, rs = ((int64_t)sib * m + fl) * B, rp = ((int64_t)par * m + fl) * B;
+  const int64_t rc = (hist_index(p, level, slot) * m + fl) * B, rs = (hist_index(p, level, sib) * m + fl) * B, rp = ((int64_t)par * m + fl) * B;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const int db = dflt ? dflt[fl] : -1;            // default bin: recovered from the node totals
   const int64_t* S = s.node_sum + h * (V + 1);

@@ -30,8 +30,10 @@ def test_sizes_and_validation_on_host():
     from paper_conf_icpp_liupw25_b200 import _abi
     P = _abi.Problem(n=2_000_000, m=4096, f_begin=0, m_global=4096, d=16, B=256, D=8, loss=0, min_node=20,
                      lambda_=1.0, gamma=0.0, lr=1.0, ld_bins=4096)
-    h, c = _abi.Context.gbdtmo_hist_bytes(P, 7)
-    assert h == 128 * 4096 * 256 * 16 * 8 and c == 128 * 4096 * 256 * 4
+    h, c = _abi.Context.gbdtmo_hist_bytes(P, 6)
+    assert h == 64 * 4096 * 256 * 16 * 8 and c == 64 * 4096 * 256 * 4
+    h, c = _abi.Context.gbdtmo_hist_bytes(P, 7)            # last level: only the built child of each pair
+    assert h == 64 * 4096 * 256 * 16 * 8 and c == 64 * 4096 * 256 * 4
     assert _abi.Context.gbdtmo_xchg_count(P) == 128 * 20 + (2_000_000 + 63) // 64
     assert _abi.Context.gbdtmo_state_bytes(P) > 3 * 4 * 2_000_000
     bad = _abi.Problem(n=10, m=4, f_begin=0, m_global=4, d=2, B=300, D=3, loss=0, min_node=1, lambda_=1.0,

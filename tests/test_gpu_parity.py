@@ -243,19 +243,26 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
         torch.cuda.synchronize()
         if sc is None:
             sc = b.scales.cpu().numpy().astype(np.float64)
-        if lvl == w.D - 1 and lvl > 0:
-            continue      # derived histograms of the last level are never materialised
-        LN = 1 << lvl
-        H = b.hist[lvl % 2][: LN * m * V * B].view(LN, m, V, B).transpose(2, 3).cpu().numpy()
-        CN = b.cnt[lvl % 2][: LN * m * B].view(LN, m, B).cpu().numpy()
+        last = lvl == w.D - 1 and lvl > 0      # derived histograms of the last level are never materialised:
+        LN = 1 << lvl                          # there only the BUILT child (the smaller, tie -> left) is checked
+        LS = LN // 2 if last else LN                      # last level: pair (2s, 2s+1) stored at slot s
+        H = b.hist[lvl % 2][: LS * m * V * B].view(LS, m, V, B).transpose(2, 3).cpu().numpy()
+        CN = b.cnt[lvl % 2][: LS * m * B].view(LS, m, B).cpu().numpy()
         for slot in range(LN):
             hid = LN - 1 + slot
             if ref["state"][0][hid] != 1:         # only nodes that were searched and split
                 continue
+            if last:
+                par = (hid - 1) // 2
+                nl, nr = ref["n_left"][0][par], ref["nrows"][0][par] - ref["n_left"][0][par]
+                built_left = nl <= nr
+                if (hid == 2 * par + 1) != built_left:
+                    continue
             r = rows[hid]
             HG, HH, CNT = orc.build_hist(bins, B, g, h, r)
-            np.testing.assert_array_equal(CN[slot], CNT)
-            gpu_g = H[slot][:, :, :d] * sc[:d]
+            hs = slot >> 1 if last else slot
+            np.testing.assert_array_equal(CN[hs], CNT)
+            gpu_g = H[hs][:, :, :d] * sc[:d]
             AG = np.zeros((m, B, d))
             np.add.at(AG, (np.arange(m)[:, None], bins[:, r]), np.abs(g[r])[None, :, :].repeat(m, 0))
             err = np.abs(gpu_g - HG) / np.maximum(np.maximum(np.abs(HG), AG), 1e-300)
@@ -263,7 +270,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
             if w.loss == 0 and w.index in (1, 3, 5):
                 assert np.array_equal(gpu_g, HG), (lvl, slot)      # dyadic tree 1: bit-exact
             if w.loss == 1:
-                gpu_h = H[slot][:, :, d:] * sc[d:]
+                gpu_h = H[hs][:, :, d:] * sc[d:]
                 assert np.all(np.abs(gpu_h - HH) <= 1e-5 * HH + CNT[:, :, None] * 2.0 ** -32)
             checked += 1
     assert checked > 0

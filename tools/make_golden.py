@@ -17,6 +17,9 @@ Contents (heap-indexed trees, NH = 2^(D+1) - 1 nodes, Algorithm 1
   nbins, cuts_digest               binning summary (nbins per feature, sha256 of the cuts bytes)
   src_sha                          sha256 of oracle.c, oracle.h, gen.py, gen.c, gen_rng.h (a test
                                    checks the goldens are not stale)
+  leaf_scale                       f64  [T][NH][d]  AG_k / (H_k + lambda) per leaf and output, AG_k = sum
+                                   |g_k| over the leaf's rows: the scale of the leaf-value error metric
+                                   (leaves inherit the histogram's |x - x*| / AG metric)
 
 usage: python tools/make_golden.py C3 [C4 C5 C2] [--T 10] [--threads N]
 """
@@ -90,13 +93,59 @@ def make(name: str, T: int) -> str:
         oracle_threads=np.array(oracle.num_threads()), seconds=np.array([t1 - t0, t2 - t1]))
     print(f"{name}: T={T} bin {t1 - t0:.1f}s train {t2 - t1:.1f}s ({oracle.num_threads()} threads) -> {out}",
           flush=True)
+    add_leaf_scale(name, T, bins=bins, Y=Y)
     return out
+
+
+def add_leaf_scale(name: str, T: int, bins=None, Y=None) -> None:
+    """Replays the golden's own trees with oracle functions only (oracle_grad at the prediction
+    before each tree, oracle_partition along the recorded splits, oracle_update_pred with the
+    recorded leaves) to get every leaf's rows, and stores leaf_scale = AG_k / (H_k + lambda)."""
+    from oracle import oracle
+    w = gen.WORKLOADS[name]
+    path = golden_path(name, T)
+    g = dict(np.load(path))
+    if bins is None:
+        _, _, bins = oracle_bins(w)
+    if Y is None:
+        X = gen.features_host(w) if w.index == 2 else None
+        Y = gen.targets_host(w, X)
+        del X
+    y = Y.astype(np.float64)
+    NH = g["state"].shape[1]
+    pred = np.zeros((w.n, w.d))
+    scale = np.zeros((T, NH, w.d))
+    for t in range(T):
+        gr, hs = oracle.grad(w.loss, y, pred)
+        rows = {0: np.arange(w.n, dtype=np.int32)}
+        st = g["state"][t]
+        for h in range(NH):
+            if h not in rows:
+                continue
+            r = rows[h]
+            if st[h] == 1:
+                left, right = oracle.partition(bins, r, int(g["feat"][t][h]), int(g["bin"][t][h]))
+                rows[2 * h + 1], rows[2 * h + 2] = left, right
+            elif st[h] == 2:
+                AG = np.abs(gr[r]).sum(0)
+                H = hs[r].sum(0)
+                scale[t, h] = AG / (H + w.lam)
+                oracle.update_pred(pred, r, g["leaf"][t][h])
+    err = float(np.max(np.abs(pred[g["sample_rows"]] - g["pred_sample"])))
+    assert err < 1e-9, f"replay of the golden's trees does not reproduce its prediction ({err})"
+    g["leaf_scale"] = scale
+    np.savez_compressed(path, **g)
+    print(f"{name}: leaf_scale added (replay matches the golden prediction to {err:.1e})", flush=True)
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("configs", nargs="+")
     ap.add_argument("--T", type=int, default=10)
+    ap.add_argument("--leaf-scale-only", action="store_true", help="add leaf_scale to existing goldens")
     a = ap.parse_args()
     for c in a.configs:
-        make(c, a.T)
+        if a.leaf_scale_only:
+            add_leaf_scale(c, a.T)
+        else:
+            make(c, a.T)

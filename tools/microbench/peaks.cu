@@ -27,7 +27,7 @@ __device__ __forceinline__ void red_add(uint32_t addr, uint32_t v) {
 }
 
 template <int MODE>
-__global__ void __launch_bounds__(1024, 1) k_atoms(int iters, int records, unsigned long long* cyc,
+__global__ void __launch_bounds__(1024, 1) k_atoms(int iters, int records, int lrec, unsigned long long* cyc,
                                                    unsigned long long* ns, unsigned* sink) {
   extern __shared__ __align__(16) uint32_t s[];
   constexpr int RW = MODE == 0 ? 32 : 192;            // words per record
@@ -44,7 +44,7 @@ __global__ void __launch_bounds__(1024, 1) k_atoms(int iters, int records, unsig
     for (int u = 0; u < 8; ++u) {
       const uint32_t h = (seed + (uint32_t)(i + u) * 0x9E3779B1u);
       // mode 1: the two half-warps take two different random records (two rows' bins)
-      const uint32_t rec = MODE == 0 ? (h >> 8) % records : ((lane < 16 ? h : (h * 0x2545F491u)) >> 8) % records;
+      const uint32_t rec = MODE == 0 ? (h >> lrec) : ((lane < 16 ? h : (h * 0x2545F491u)) >> lrec);
       red_add(base + 4u * (rec * RW + lanew), (uint32_t)u + 1u);
     }
   }
@@ -73,7 +73,8 @@ extern "C" int peaks_atoms(int device, int mode, int iters, double* lane_ops_per
   int sms = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
   const int RW = mode == 0 ? 32 : 192;
-  const int records = (200 * 1024) / (4 * RW);
+  const int records = mode == 0 ? 1024 : 256;            // 128 KB / 192 KB, a power of two
+  const int lrec = mode == 0 ? 22 : 24;                  // record = top log2(records) bits of a hash
   const int smem = records * RW * 4;
   unsigned long long *cyc = nullptr, *ns = nullptr;
   unsigned* sink = nullptr;
@@ -84,7 +85,7 @@ extern "C" int peaks_atoms(int device, int mode, int iters, double* lane_ops_per
     auto kern = mode == 0 ? k_atoms<0> : k_atoms<1>;
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     for (int rep = 0; rep < 2 && e == cudaSuccess; ++rep) {        // rep 0: warm-up
-      kern<<<sms, 1024, smem>>>(iters, records, cyc, ns, sink);
+      kern<<<sms, 1024, smem>>>(iters, records, lrec, cyc, ns, sink);
       e = cudaDeviceSynchronize();
     }
   }

@@ -303,10 +303,16 @@ gbdtmo_status gbdtmo_partition(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t 
 /* ------------------------------------------------------------ (a)8, (a)9 */
 
 /* Leaf values: for every heap node in state LEAF,
- *   leaf[h][k] = -lr * G_k / (H_k + lambda)   (G, H = exact node sums, MSE: H = 2 * count);
- * other heap nodes get 0.  leaf float64 [2^(D+1)-1][d]. */
-gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* scales,
-                                 void* state, double* leaf);
+ *   leaf[h][k] = -lr * G_k / (H_k + lambda)         (MSE: H = 2 * count);
+ * other heap nodes get 0.  leaf float64 [2^(D+1)-1][d].
+ * With y and pred (the tree's targets and PRE-tree prediction, as given to gbdtmo_grad; call before
+ * gbdtmo_update_pred): G, H are fp64 sums of g, h recomputed in fp64 over the leaf's rows (reading
+ * R17), in a fixed order (deterministic, identical on every rank) -- the oracle's definition up to
+ * summation order.  With y = pred = NULL: G, H from the exact fixed-point node sums (scales from
+ * gbdtmo_grad), whose absolute resolution is n_leaf P 2^-31 (R29). */
+gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* scales, void* state,
+                                 const float* y /* may be NULL */, const double* pred /* may be NULL */,
+                                 double* leaf);
 
 /* Incremental prediction (rows read their leaf directly, no traversal):
  *   pred[i][k] += leaf[node_of(i)][k]   for every instance i.   pred float64 [n][d] in/out

@@ -86,7 +86,7 @@ def lib():
             "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_search_small": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
-            "gbdtmo_leaf_values": ([P, PP, P, P, P], C.c_int),
+            "gbdtmo_leaf_values": ([P, PP, P, P, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_predict": ([P, P, i64, i32, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
@@ -241,8 +241,9 @@ class Context:
         self._check(lib().gbdtmo_partition(self._h, C.byref(p), level, _ptr(state), _ptr(xchg)),
                     "gbdtmo_partition")
 
-    def gbdtmo_leaf_values(self, p, scales, state, leaf):
-        self._check(lib().gbdtmo_leaf_values(self._h, C.byref(p), _ptr(scales), _ptr(state), _ptr(leaf)),
+    def gbdtmo_leaf_values(self, p, scales, state, leaf, y=None, pred=None):
+        self._check(lib().gbdtmo_leaf_values(self._h, C.byref(p), _ptr(scales), _ptr(state), _ptr(y), _ptr(pred),
+                                             _ptr(leaf)),
                     "gbdtmo_leaf_values")
 
     def gbdtmo_update_pred(self, p, state, leaf, pred):

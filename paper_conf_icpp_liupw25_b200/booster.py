@@ -416,7 +416,7 @@ class Booster:
                 # (plumbing: one device copy per dataset) the level-0 counts after find_split
                 self.root_cnt = self.cnt[0][: self.p.m * self.p.B].clone()
         self._mark("leaf+update", time_hist)
-        ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf)
+        ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf, self.y, self.pred)   # fp64 sums (R17)
         ctx.gbdtmo_update_pred(p, self.state, self.leaf, self.pred)
         self._mark("end", time_hist)
         if time_hist:

@@ -23,6 +23,86 @@ __global__ void k_leaf_values(gbdtmo_problem p, const float* __restrict__ scales
   }
 }
 
+// Leaf values from fp64 node totals summed from the leaf's rows (reading R17; the oracle's
+// definition), not from the 31-bit fixed-point sums: g, h are recomputed in fp64 from y and the
+// pre-tree prediction exactly as gbdtmo_grad computes them before quantising, so a leaf whose rows
+// all have tiny |g| (confident softmax rows: G ~ 1e-3, quantisation floor n 2^-31) is exact to fp64
+// rounding instead of to the fixed point's absolute resolution.  One block per heap node (LEAF
+// only); warp w sums a fixed contiguous part of the leaf's segment of the final row list in row
+// order, lanes over channels; the 8 warps' partials are combined in warp order: deterministic and
+// identical on every rank (replicated rows and predictions).
+constexpr int kLeafWarps = 8;
+constexpr int kLeafChunk = 256;          // channels per pass (8 fp64 accumulators per lane)
+
+__global__ void __launch_bounds__(kLeafWarps * 32)
+k_leaf_values_exact(gbdtmo_problem p, const float* __restrict__ y, const double* __restrict__ pred, State s,
+                    double* __restrict__ leaf) {
+  extern __shared__ double lsm[];                       // [V] totals, then [kLeafWarps][kLeafChunk] partials
+  const int64_t h = blockIdx.x;
+  const int d = p.d, V = channels(p);
+  const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
+  if (s.node_state[h] != GBDTMO_NODE_LEAF) {
+    for (int k = threadIdx.x; k < d; k += blockDim.x) leaf[h * d + k] = 0.0;
+    return;
+  }
+  double* tot = lsm;
+  double* part = lsm + V;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int32_t* rl = (p.D & 1) ? s.rows1 : s.rows0;    // the list after the last level's partition
+  const int64_t b = s.node_begin[h], e = s.node_end[h];
+  const int64_t per = (e - b + kLeafWarps - 1) / kLeafWarps;
+  const int64_t wb = b + warp * per, we = min(e, wb + per);
+  for (int c0 = 0; c0 < V; c0 += kLeafChunk) {
+    double acc[kLeafChunk / 32];
+#pragma unroll
+    for (int u = 0; u < kLeafChunk / 32; ++u) acc[u] = 0.0;
+    for (int64_t pos = wb; pos < we; ++pos) {
+      const int64_t i = rl[pos];
+      const double* pr = pred + i * d;
+      const float* yr = y + i * d;
+      double mx = -INFINITY, z = 0.0;
+      if (softmax) {                                     // p = softmax(yhat_i) (max-subtracted), R12
+        for (int k = lane; k < d; k += 32) mx = fmax(mx, pr[k]);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        for (int k = lane; k < d; k += 32) z += exp(pr[k] - mx);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
+      }
+#pragma unroll
+      for (int u = 0; u < kLeafChunk / 32; ++u) {
+        const int c = c0 + u * 32 + lane;
+        if (c < V) {
+          double v;
+          if (!softmax) {
+            v = 2.0 * (pr[c] - (double)yr[c]);           // g = 2 (yhat - y)
+          } else {
+            const int k = c < d ? c : c - d;
+            const double pk = exp(pr[k] - mx) / z;
+            v = c < d ? pk - (double)yr[k] : pk * (1.0 - pk);   // g = p - y, h = p (1 - p)
+          }
+          acc[u] += v;
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kLeafChunk / 32; ++u) part[warp * kLeafChunk + u * 32 + lane] = acc[u];
+    __syncthreads();
+    for (int c = threadIdx.x; c < kLeafChunk && c0 + c < V; c += blockDim.x) {
+      double t = 0.0;
+      for (int w = 0; w < kLeafWarps; ++w) t += part[w * kLeafChunk + c];
+      tot[c0 + c] = t;
+    }
+    __syncthreads();
+  }
+  const double cntd = (double)s.node_sum[h * (V + 1) + V];
+  for (int k = threadIdx.x; k < d; k += blockDim.x) {
+    const double G = tot[k];
+    const double H = softmax ? tot[d + k] : 2.0 * cntd;  // MSE: h = 2 for every row
+    leaf[h * d + k] = -p.lr * G / (H + p.lambda);
+  }
+}
+
 // pred[i][k] += leaf[nid[i]][k]: every instance reads its leaf directly (no traversal).
 __global__ void k_update_pred(gbdtmo_problem p, State s, const double* __restrict__ leaf, double* __restrict__ pred) {
   const int d = p.d;
@@ -172,15 +252,24 @@ extern "C" gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx c, const gbdtmo_problem* 
 }
 
 extern "C" gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx c, const gbdtmo_problem* p, const float* scales,
-                                            void* state, double* leaf) {
+                                            void* state, const float* y, const double* pred, double* leaf) {
   Ctx* ctx = (Ctx*)c;
   DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
-  GB_CHECK_ARG(scales && state && leaf, "null pointer");
+  GB_CHECK_ARG(state && leaf, "null pointer");
+  GB_CHECK_ARG((y == nullptr) == (pred == nullptr), "y and pred must be given together");
   State s = state_view(*p, state);
-  GB_LAUNCH(k_leaf_values, 64, 256, 0, *p, scales, s, leaf);
+  if (y) {
+    const int smem = (channels(*p) + kLeafWarps * kLeafChunk) * 8;
+    static unsigned long long attr_mask = 0;
+    smem_optin_once(ctx, k_leaf_values_exact, attr_mask, ctx->max_smem_optin - 1024);
+    GB_LAUNCH(k_leaf_values_exact, (unsigned)heap_nodes(*p), kLeafWarps * 32, smem, *p, y, pred, s, leaf);
+  } else {
+    GB_CHECK_ARG(scales, "null scales");
+    GB_LAUNCH(k_leaf_values, 64, 256, 0, *p, scales, s, leaf);
+  }
   return GBDTMO_OK;
 }
 

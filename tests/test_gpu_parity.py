@@ -379,7 +379,7 @@ def test_two_shards_equal_one(orc, pkg, ctx):
                 s.xchg.copy_(xs)
                 ctx.gbdtmo_partition(s.p, lvl, s.state, s.xchg)
         for s in shards:
-            ctx.gbdtmo_leaf_values(s.p, s.scales, s.state, s.leaf)
+            ctx.gbdtmo_leaf_values(s.p, s.scales, s.state, s.leaf, s.y, s.pred)
             ctx.gbdtmo_update_pred(s.p, s.state, s.leaf, s.pred)
             s.trees.append(s.export())
     torch.cuda.synchronize()
@@ -496,3 +496,31 @@ def test_packed_bins_layout_and_equivalence(orc, pkg, ctx, case, sparse):
             np.testing.assert_array_equal(a[key], b[key])
         assert not compare_trees(a, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t])
     assert np.max(np.abs(bp.pred.cpu().numpy() - ref["pred"])) <= 1e-4
+
+
+@pytest.mark.parametrize("case", ["C2s", "C3s", "S300s"])
+def test_leaf_values_fp64_exact_vs_fixed_point(orc, pkg, ctx, case):
+    """gbdtmo_leaf_values with y / pred sums g, h in fp64 over each leaf's rows (R17): the leaves equal
+    the oracle's to fp64 rounding (rtol 1e-10 + 1e-13), also for confident softmax leaves whose tiny G
+    sits at the fixed point's resolution floor n_leaf 2^-31 (R29); the fixed-point path
+    (y = pred = NULL) stays within that floor of them."""
+    w = CASES[case].scaled(T=4)
+    X, Y = _inputs(w)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B), torch.from_numpy(Y).to(DEV),
+                    _params(pkg, w))
+    for t in range(w.T):
+        b._tree()                                    # leaf values from fp64 row sums (the default)
+        torch.cuda.synchronize()
+        fixed = torch.empty_like(b.leaf)
+        # (the prediction has been updated: recompute the fixed-point leaves from the same state)
+        ctx.gbdtmo_leaf_values(b.p, b.scales, b.state, fixed)
+        torch.cuda.synchronize()
+        rec = to_np(b.export())
+        assert not compare_trees(rec, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t])
+        lv = rec["node_state"] == 2
+        np.testing.assert_allclose(rec["leaf"][lv], ref["leaf"][t][lv], rtol=1e-10, atol=1e-13)
+        floor = rec["n_rows"][lv][:, None] * 2.0 ** -30 / w.lam * (1 if w.loss == 1 else 64)
+        assert np.all(np.abs(fixed.cpu().numpy()[lv] - rec["leaf"][lv]) <= floor + 1e-9 * np.abs(rec["leaf"][lv]))

@@ -9,7 +9,9 @@
 // mode 1  the histogram kernel's lane map (hist.cu, K = 16): lanes 0-15 add to words c of a
 //         random 192-word bin record, lanes 16-31 to words 16 + c of another random record (the
 //         swapped-limb row pair), i.e. the exact address pattern of one k_hist_smem instruction.
-// Both: 1024 threads x 1 CTA per SM, ~200 KB of shared memory, U = 8 atomics in flight per
+// mode 2  a row-per-instruction lane map (proposal): all 32 lanes add to the 32 words (16 lo + 16 hi
+//         limbs) of ONE random 32-word feature slot of a random 192-word bin record.
+// All: 1024 threads x 1 CTA per SM, ~200 KB of shared memory, U = 8 atomics in flight per
 // thread; cycles from clock64 (max over CTAs), time from %globaltimer.
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -31,6 +33,7 @@ __global__ void __launch_bounds__(1024, 1) k_atoms(int iters, int records, int l
                                                    unsigned long long* ns, unsigned* sink) {
   extern __shared__ __align__(16) uint32_t s[];
   constexpr int RW = MODE == 0 ? 32 : 192;            // words per record
+  static_assert(MODE >= 0 && MODE <= 2, "mode");
   for (int i = threadIdx.x; i < records * RW; i += blockDim.x) s[i] = 0;
   __syncthreads();
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -44,8 +47,9 @@ __global__ void __launch_bounds__(1024, 1) k_atoms(int iters, int records, int l
     for (int u = 0; u < 8; ++u) {
       const uint32_t h = (seed + (uint32_t)(i + u) * 0x9E3779B1u);
       // mode 1: the two half-warps take two different random records (two rows' bins)
-      const uint32_t rec = MODE == 0 ? (h >> lrec) : ((lane < 16 ? h : (h * 0x2545F491u)) >> lrec);
-      red_add(base + 4u * (rec * RW + lanew), (uint32_t)u + 1u);
+      const uint32_t rec = MODE == 1 ? ((lane < 16 ? h : (h * 0x2545F491u)) >> lrec) : (h >> lrec);
+      const uint32_t jw = MODE == 2 ? 32u * ((uint32_t)(i + u) % 6u) : 0u;
+      red_add(base + 4u * (rec * RW + jw + lanew), (uint32_t)u + 1u);
     }
   }
   __syncthreads();
@@ -75,6 +79,7 @@ extern "C" int peaks_atoms(int device, int mode, int iters, double* lane_ops_per
   const int RW = mode == 0 ? 32 : 192;
   const int records = mode == 0 ? 1024 : 256;            // 128 KB / 192 KB, a power of two
   const int lrec = mode == 0 ? 22 : 24;                  // record = top log2(records) bits of a hash
+  if (mode < 0 || mode > 2) return (int)cudaErrorInvalidValue;
   const int smem = records * RW * 4;
   unsigned long long *cyc = nullptr, *ns = nullptr;
   unsigned* sink = nullptr;
@@ -82,7 +87,7 @@ extern "C" int peaks_atoms(int device, int mode, int iters, double* lane_ops_per
   if (e == cudaSuccess) e = cudaMalloc(&sink, 4);
   if (e == cudaSuccess) {
     ns = cyc + sms;
-    auto kern = mode == 0 ? k_atoms<0> : k_atoms<1>;
+    auto kern = mode == 0 ? k_atoms<0> : mode == 1 ? k_atoms<1> : k_atoms<2>;
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     for (int rep = 0; rep < 2 && e == cudaSuccess; ++rep) {        // rep 0: warm-up
       kern<<<sms, 1024, smem>>>(iters, records, lrec, cyc, ns, sink);

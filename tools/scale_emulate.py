@@ -112,7 +112,7 @@ def tree(ranks, D):
         run(lambda b, lvl=lvl: b.ctx.gbdtmo_partition(b.p, lvl, b.state, b.xchg), f"L{lvl} partition")
 
     def fin(b):
-        b.ctx.gbdtmo_leaf_values(b.p, b.scales, b.state, b.leaf)
+        b.ctx.gbdtmo_leaf_values(b.p, b.scales, b.state, b.leaf, b.y, b.pred)
         b.ctx.gbdtmo_update_pred(b.p, b.state, b.leaf, b.pred)
     run(fin, "leaf+update")
     return phases

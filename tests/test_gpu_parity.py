@@ -522,5 +522,8 @@ def test_leaf_values_fp64_exact_vs_fixed_point(orc, pkg, ctx, case):
         assert not compare_trees(rec, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t])
         lv = rec["node_state"] == 2
         np.testing.assert_allclose(rec["leaf"][lv], ref["leaf"][t][lv], rtol=1e-10, atol=1e-13)
-        floor = rec["n_rows"][lv][:, None] * 2.0 ** -30 / w.lam * (1 if w.loss == 1 else 64)
+        # |dG| <= n P_g 2^-31, |dH| <= n P_h 2^-31 (softmax P_g = 1, P_h = 1/4; MSE H is exact) ->
+        # |dv| <= (|dG| + |v| |dH|) / lambda
+        pg = 1.0 if w.loss == 1 else 64.0
+        floor = rec["n_rows"][lv][:, None] * 2.0 ** -31 * (pg + np.abs(rec["leaf"][lv])) / w.lam * 2
         assert np.all(np.abs(fixed.cpu().numpy()[lv] - rec["leaf"][lv]) <= floor + 1e-9 * np.abs(rec["leaf"][lv]))

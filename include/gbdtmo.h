@@ -192,10 +192,12 @@ gbdtmo_status gbdtmo_default_bins(gbdtmo_ctx ctx, const uint8_t* bins, int64_t n
  *   pred   float64 [n][d]   current prediction yhat (sum of previous trees)
  *   q      int32   [n][V]   out: q[i][c] (MSE: g; softmax: g for c < d, h for c >= d)
  *   scales float32 [V]      out: dequantisation factor P_c * 2^-30 (a power of two)
+ *   gh     float64 [n][V]   out, may be NULL: the fp64 g (and softmax h) before quantisation, for
+ *                           gbdtmo_leaf_values' fp64 leaf sums
  *   state  gbdtmo_state_bytes(p) bytes, out: root node = all rows (sums of q = exact int64),
  *          per-row node ids = root, level-0 build plan. */
 gbdtmo_status gbdtmo_grad(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* y, const double* pred,
-                          int32_t* q, float* scales, void* state);
+                          int32_t* q, float* scales, void* state, double* gh /* may be NULL */);
 
 /* ------------------------------------------------------ (a)3 histogram build */
 
@@ -305,14 +307,12 @@ gbdtmo_status gbdtmo_partition(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t 
 /* Leaf values: for every heap node in state LEAF,
  *   leaf[h][k] = -lr * G_k / (H_k + lambda)         (MSE: H = 2 * count);
  * other heap nodes get 0.  leaf float64 [2^(D+1)-1][d].
- * With y and pred (the tree's targets and PRE-tree prediction, as given to gbdtmo_grad; call before
- * gbdtmo_update_pred): G, H are fp64 sums of g, h recomputed in fp64 over the leaf's rows (reading
- * R17), in a fixed order (deterministic, identical on every rank) -- the oracle's definition up to
- * summation order.  With y = pred = NULL: G, H from the exact fixed-point node sums (scales from
+ * With gh (gbdtmo_grad's fp64 g / h of this tree): G, H are fp64 sums over the leaf's rows (reading
+ * R17) in a fixed order (deterministic, identical on every rank) -- the oracle's definition up to
+ * summation order.  With gh = NULL: G, H from the exact fixed-point node sums (scales from
  * gbdtmo_grad), whose absolute resolution is n_leaf P 2^-31 (R29). */
 gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx ctx, const gbdtmo_problem* p, const float* scales, void* state,
-                                 const float* y /* may be NULL */, const double* pred /* may be NULL */,
-                                 double* leaf);
+                                 const double* gh /* may be NULL */, double* leaf);
 
 /* Incremental prediction (rows read their leaf directly, no traversal):
  *   pred[i][k] += leaf[node_of(i)][k]   for every instance i.   pred float64 [n][d] in/out

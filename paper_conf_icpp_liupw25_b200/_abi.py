@@ -76,7 +76,7 @@ def lib():
             "gbdtmo_xchg_count": ([PP, C.POINTER(i64)], C.c_int),
             "gbdtmo_bin": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz], C.c_int),
             "gbdtmo_bin_csc": ([P, P, P, P, P, i64, i32, i32, P, i64, P, P, P, sz], C.c_int),
-            "gbdtmo_grad": ([P, PP, P, P, P, P, P], C.c_int),
+            "gbdtmo_grad": ([P, PP, P, P, P, P, P, P], C.c_int),
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_build_hist_packed": ([P, PP, i32, P, P, P, P, P, P, P], C.c_int),
@@ -86,7 +86,7 @@ def lib():
             "gbdtmo_split_record": ([P, PP, i32, P, P, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_search_small": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_partition": ([P, PP, i32, P, P], C.c_int),
-            "gbdtmo_leaf_values": ([P, PP, P, P, P, P, P], C.c_int),
+            "gbdtmo_leaf_values": ([P, PP, P, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
             "gbdtmo_predict": ([P, P, i64, i32, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
@@ -197,9 +197,9 @@ class Context:
         self._check(lib().gbdtmo_bin(self._h, _ptr(X), n, m, ld_x, B, _ptr(bins), ld_bins, _ptr(cuts),
                                      _ptr(nbins), _ptr(ws), ws_bytes), "gbdtmo_bin")
 
-    def gbdtmo_grad(self, p, y, pred, q, scales, state):
+    def gbdtmo_grad(self, p, y, pred, q, scales, state, gh=None):
         self._check(lib().gbdtmo_grad(self._h, C.byref(p), _ptr(y), _ptr(pred), _ptr(q), _ptr(scales),
-                                      _ptr(state)), "gbdtmo_grad")
+                                      _ptr(state), _ptr(gh)), "gbdtmo_grad")
 
     def gbdtmo_default_bins(self, bins, n, m, ld_bins, B, min_count, dflt):
         self._check(lib().gbdtmo_default_bins(self._h, _ptr(bins), n, m, ld_bins, B, min_count, _ptr(dflt)),
@@ -241,9 +241,8 @@ class Context:
         self._check(lib().gbdtmo_partition(self._h, C.byref(p), level, _ptr(state), _ptr(xchg)),
                     "gbdtmo_partition")
 
-    def gbdtmo_leaf_values(self, p, scales, state, leaf, y=None, pred=None):
-        self._check(lib().gbdtmo_leaf_values(self._h, C.byref(p), _ptr(scales), _ptr(state), _ptr(y), _ptr(pred),
-                                             _ptr(leaf)),
+    def gbdtmo_leaf_values(self, p, scales, state, leaf, gh=None):
+        self._check(lib().gbdtmo_leaf_values(self._h, C.byref(p), _ptr(scales), _ptr(state), _ptr(gh), _ptr(leaf)),
                     "gbdtmo_leaf_values")
 
     def gbdtmo_update_pred(self, p, state, leaf, pred):

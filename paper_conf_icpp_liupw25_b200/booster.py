@@ -234,6 +234,7 @@ class Booster:
         self.pred = pred if pred is not None else torch.zeros((n, d), dtype=torch.float64, device=dev)
         assert self.pred.dtype == torch.float64
         self.q = torch.empty((n, V), dtype=torch.int32, device=dev)
+        self.gh = torch.empty((n, V), dtype=torch.float64, device=dev)   # fp64 g/h for exact leaf sums
         self.scales = torch.empty(V, dtype=torch.float32, device=dev)
         self.state = torch.empty(ctx.gbdtmo_state_bytes(self.p), dtype=torch.uint8, device=dev)
         self.hist, self.cnt = [None, None], [None, None]
@@ -408,7 +409,7 @@ class Booster:
         self._apply_options()
         self._marks = []
         self._mark("grad", time_hist)
-        ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state)
+        ctx.gbdtmo_grad(p, self.y, self.pred, self.q, self.scales, self.state, self.gh)
         for lvl in range(self.params.D):
             self._mark("build_hist", time_hist)
             self._level(lvl, time_hist)
@@ -416,7 +417,7 @@ class Booster:
                 # (plumbing: one device copy per dataset) the level-0 counts after find_split
                 self.root_cnt = self.cnt[0][: self.p.m * self.p.B].clone()
         self._mark("leaf+update", time_hist)
-        ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf, self.y, self.pred)   # fp64 sums (R17)
+        ctx.gbdtmo_leaf_values(p, self.scales, self.state, self.leaf, self.gh)   # fp64 row sums (R17)
         ctx.gbdtmo_update_pred(p, self.state, self.leaf, self.pred)
         self._mark("end", time_hist)
         if time_hist:

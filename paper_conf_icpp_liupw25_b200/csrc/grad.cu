@@ -47,7 +47,7 @@ __device__ __forceinline__ int pow2_exponent(double S) {
 
 // MSE pass 2: q = rint(g * 2^(30 - log2 P)), exact root sums.  block (32, 8): x = channel, y = row.
 __global__ void k_mse_quantize(gbdtmo_problem p, const float* __restrict__ y, const double* __restrict__ pred,
-                               int32_t* __restrict__ q, float* __restrict__ scales, State s) {
+                               int32_t* __restrict__ q, float* __restrict__ scales, State s, double* __restrict__ gh) {
   __shared__ long long red[8][33];
   const int d = p.d;
   for (int c0 = 0; c0 < d; c0 += 32) {
@@ -58,6 +58,7 @@ __global__ void k_mse_quantize(gbdtmo_problem p, const float* __restrict__ y, co
     if (on) {
       for (int64_t i = blockIdx.x * 8 + threadIdx.y; i < p.n; i += (int64_t)gridDim.x * 8) {
         const double g = 2.0 * (pred[i * d + c] - (double)y[i * d + c]);
+        if (gh) gh[i * d + c] = g;                      // fp64 g for the leaf values (R17)
         const int qi = __double2int_rn(ldexp(g, kQShift - ex));
         q[i * d + c] = qi;
         acc += qi;
@@ -79,7 +80,8 @@ __global__ void k_mse_quantize(gbdtmo_problem p, const float* __restrict__ y, co
 // q_g = rint(g 2^30) (P = 1), q_h = rint(h 2^32) (P = 1/4).  Any d (lanes stride the outputs;
 // exp is recomputed instead of held in registers).
 __global__ void k_softmax_quantize(gbdtmo_problem p, const float* __restrict__ y, const double* __restrict__ pred,
-                                   int32_t* __restrict__ q, float* __restrict__ scales, State s) {
+                                   int32_t* __restrict__ q, float* __restrict__ scales, State s,
+                                   double* __restrict__ gh) {
   const int d = p.d, V = 2 * d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   for (int64_t i = blockIdx.x * (int64_t)nw + warp; i < p.n; i += (int64_t)gridDim.x * nw) {
@@ -98,6 +100,7 @@ __global__ void k_softmax_quantize(gbdtmo_problem p, const float* __restrict__ y
       const double h = pk * (1.0 - pk);
       q[i * V + c] = __double2int_rn(ldexp(g, kQShift));
       q[i * V + d + c] = __double2int_rn(ldexp(h, kQShift + 2));
+      if (gh) { gh[i * V + c] = g; gh[i * V + d + c] = h; }   // fp64 g, h for the leaf values (R17)
     }
   }
   if (blockIdx.x == 0) {
@@ -165,7 +168,7 @@ int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p) {
 using namespace gbdtmo;
 
 extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, const float* y, const double* pred,
-                                     int32_t* q, float* scales, void* state) {
+                                     int32_t* q, float* scales, void* state, double* gh) {
   Ctx* ctx = (Ctx*)c;
   DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
@@ -177,9 +180,9 @@ extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, cons
   GB_LAUNCH(k_tree_reset, sms, 256, 0, *p, s);
   if (p->loss == GBDTMO_LOSS_MSE) {
     GB_LAUNCH(k_mse_max, sms * 4, dim3(32, 8), 0, *p, y, pred, s);
-    GB_LAUNCH(k_mse_quantize, sms * 4, dim3(32, 8), 0, *p, y, pred, q, scales, s);
+    GB_LAUNCH(k_mse_quantize, sms * 4, dim3(32, 8), 0, *p, y, pred, q, scales, s, gh);
   } else {
-    GB_LAUNCH(k_softmax_quantize, sms * 4, 256, 0, *p, y, pred, q, scales, s);
+    GB_LAUNCH(k_softmax_quantize, sms * 4, 256, 0, *p, y, pred, q, scales, s, gh);
     GB_LAUNCH(k_qsum, sms * 4, dim3(32, 8), 0, *p, q, s);
   }
   GB_LAUNCH(k_rows_init, sms * 4, 256, 0, *p, s);

@@ -72,14 +72,6 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #define GBDTMO_HIST_SHFL 0         // (A/B) 1: phase 2 takes the bins by SHFL, no scratch round trip
 #endif
   constexpr int SB = G < GBDTMO_HIST_SB ? G : GBDTMO_HIST_SB;   // groups per q-prefetch sub-batch
-#ifndef GBDTMO_HIST_ROW1
-#define GBDTMO_HIST_ROW1 1        // K = 16: one row per instruction (lo | hi limbs of 16 channels)
-#endif
-  constexpr bool ROW1 = GBDTMO_HIST_ROW1 && K == 16 && !GBDTMO_HIST_LCNT;
-#ifndef GBDTMO_HIST_SB1
-#define GBDTMO_HIST_SB1 4         // ROW1: rows of q prefetched ahead
-#endif
-  constexpr int SB1 = GBDTMO_HIST_SB1;
   constexpr int RS = KF * 2 * K;               // limb words per bin
   constexpr int NW = PACKED ? 1 : HistRow<KF>::NW, SW = PACKED ? 1 : HistRow<KF>::SW;
   static_assert(!PACKED || KF <= 8, "packed tiles hold <= 8 features");
@@ -101,9 +93,6 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
   // limb selectors for PRMT(q, sel, 0): lo = bytes 0-1 zero-extended (0x4410), hi = bytes 2-3
   // sign-extended (0xBB32); even rows add (lo, hi) at (slotA, slotB), odd rows (hi, lo)
   const uint32_t selA = (ri & 1) ? 0xBB32u : 0x4410u, selB = (ri & 1) ? 0x4410u : 0xBB32u;
-  // ROW1 lanes: channel c = lane % 16 (as above), limb lane / 16 (0: lo at word c, 1: hi at word 16 + c)
-  const uint32_t sel1 = (lane < 16) ? 0x4410u : 0xBB32u;
-  const uint32_t a1 = sbase + 4u * lane;
   // lane counts (LCNT): lane (ri, c < 2 KF) counts feature cj of the earlier (c < KF) or later
   // row pair of every two, into column 16 ri + c of the [bin/2][32] table (bank = column)
   const int cj = c < KF ? c : c - KF;
@@ -160,13 +149,6 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
         qv[t] = (rr >= 0 && chan_on) ? __ldg(qc + (int64_t)rr * V) : 0;
       }
     };
-    auto load_q1 = [&](int rid, int t0, int (&qv)[SB1]) {
-#pragma unroll
-      for (int t = 0; t < SB1; ++t) {
-        const int rr = __shfl_sync(0xffffffffu, rid, t0 + t);
-        qv[t] = (rr >= 0 && chan_on) ? __ldg(qc + (int64_t)rr * V) : 0;
-      }
-    };
     int r_cur = load_rid(beg + warp * 32 + lane);
     int r_nxt = load_rid(beg + warp * 32 + bstep + lane);
 #if GBDTMO_HIST_WDEPTH == 2
@@ -176,10 +158,8 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #endif
     uint64_t w_cur[NW];
     load_win(r_cur, w_cur);
-    int qv[ROW1 ? 1 : SB];
-    int q1[ROW1 ? SB1 : 1];
-    if constexpr (ROW1) load_q1(r_cur, 0, q1);
-    else load_q(r_cur, 0, qv);
+    int qv[SB];
+    load_q(r_cur, 0, qv);
     for (int b0 = beg + warp * 32; b0 < end; b0 += bstep) {
 #if GBDTMO_HIST_WDEPTH == 2
       // (gathered deep levels) bin windows two batches ahead, row ids three
@@ -226,77 +206,49 @@ k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, cons
 #pragma unroll
       for (int i = 0; i < SW; ++i) scratch[lane * SW + i] = sw[i];
       __syncwarp();
-      // ---- phase 2
-      if constexpr (ROW1) {
-        // one row per warp instruction: lanes 0-15 add the lo limbs of the row's 16 channels,
-        // lanes 16-31 the hi limbs, all into the same 32-word (128-byte) record of (bin, feature):
-        // one shared line per instruction (tools/microbench/peaks.cu mode 2 vs mode 1)
-#pragma unroll 1
-        for (int t0 = 0; t0 < 32; t0 += SB1) {
-          int qn[SB1];
-          if (t0 + SB1 < 32) load_q1(r, t0 + SB1, qn);
-          else load_q1(r_nxt, 0, qn);
+      // ---- phase 2: groups of RPI rows x K channels
+      const bool cnt_on = LCNT && do_cnt && c < 2 * KF && cj < kk;
+      uint64_t bprev = 0;
 #pragma unroll
-          for (int t = 0; t < SB1; ++t) {
-            const int i = t0 + t;
-            uint64_t bw[SW];
+      for (int t0 = 0; t0 < G; t0 += SB) {
+        int qn[SB];
+        if (t0 + SB < G) load_q(r, t0 + SB, qn);
+        else load_q(r_nxt, 0, qn);
+#pragma unroll
+        for (int t = 0; t < SB; ++t) {
+          const int i = (t0 + t) * RPI + ri;
+          uint64_t bw[SW];
+          if (GBDTMO_HIST_SHFL && SW == 1) {       // (A/B) bins by shuffle instead of the scratch
+            const uint32_t w0 = __shfl_sync(0xffffffffu, (uint32_t)sw[0], i);
+            const uint32_t w1 = KF > 4 ? __shfl_sync(0xffffffffu, (uint32_t)(sw[0] >> 32), i) : 0u;
+            bw[0] = ((uint64_t)w1 << 32) | w0;
+          } else {
 #pragma unroll
             for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
-            const uint32_t v = prmt_sx((uint32_t)q1[t], sel1);
+          }
+          if (LCNT) {
+            if ((t0 + t) & 1) {
+              const uint64_t w = c < KF ? bprev : bw[0];
+              const int row = c < KF ? i - 2 : i;
+              const uint32_t bin = (uint32_t)(w >> cshift) & 0xFFu;
+              if (cnt_on && b0 + row < end && (!SKIP || (int)bin != dfl_of(dfl, cj)))
+                red_shared_add(acol + (bin >> 1) * 128u, 1u << ((bin & 1) << 4));
+            }
+            bprev = bw[0];
+          }
+          const uint32_t va = prmt_sx((uint32_t)qv[t], selA);
+          const uint32_t vb = prmt_sx((uint32_t)qv[t], selB);
 #pragma unroll
-            for (int j = 0; j < KF; ++j) {
-              const uint32_t bin = byte_of<SW>(bw, j);
-              if (!SKIP || (int)bin != dfl[j]) red_shared_add(a1 + bin * (4u * RS) + 8u * K * j, v);
+          for (int j = 0; j < KF; ++j) {
+            const uint32_t bin = byte_of<SW>(bw, j);
+            if (!SKIP || (int)bin != dfl[j]) {
+              red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
+              red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
             }
           }
+        }
 #pragma unroll
-          for (int t = 0; t < SB1; ++t) q1[t] = qn[t];
-        }
-      } else {
-      // ---- phase 2: groups of RPI rows x K channels
-        const bool cnt_on = LCNT && do_cnt && c < 2 * KF && cj < kk;
-        uint64_t bprev = 0;
-  #pragma unroll
-        for (int t0 = 0; t0 < G; t0 += SB) {
-          int qn[SB];
-          if (t0 + SB < G) load_q(r, t0 + SB, qn);
-          else load_q(r_nxt, 0, qn);
-  #pragma unroll
-          for (int t = 0; t < SB; ++t) {
-            const int i = (t0 + t) * RPI + ri;
-            uint64_t bw[SW];
-            if (GBDTMO_HIST_SHFL && SW == 1) {       // (A/B) bins by shuffle instead of the scratch
-              const uint32_t w0 = __shfl_sync(0xffffffffu, (uint32_t)sw[0], i);
-              const uint32_t w1 = KF > 4 ? __shfl_sync(0xffffffffu, (uint32_t)(sw[0] >> 32), i) : 0u;
-              bw[0] = ((uint64_t)w1 << 32) | w0;
-            } else {
-  #pragma unroll
-              for (int u = 0; u < SW; ++u) bw[u] = scratch[i * SW + u];
-            }
-            if (LCNT) {
-              if ((t0 + t) & 1) {
-                const uint64_t w = c < KF ? bprev : bw[0];
-                const int row = c < KF ? i - 2 : i;
-                const uint32_t bin = (uint32_t)(w >> cshift) & 0xFFu;
-                if (cnt_on && b0 + row < end && (!SKIP || (int)bin != dfl_of(dfl, cj)))
-                  red_shared_add(acol + (bin >> 1) * 128u, 1u << ((bin & 1) << 4));
-              }
-              bprev = bw[0];
-            }
-            const uint32_t va = prmt_sx((uint32_t)qv[t], selA);
-            const uint32_t vb = prmt_sx((uint32_t)qv[t], selB);
-  #pragma unroll
-            for (int j = 0; j < KF; ++j) {
-              const uint32_t bin = byte_of<SW>(bw, j);
-              if (!SKIP || (int)bin != dfl[j]) {
-                red_shared_add(aA + bin * (4u * RS) + 8u * K * j, va);
-                red_shared_add(aB + bin * (4u * RS) + 8u * K * j, vb);
-              }
-            }
-          }
-  #pragma unroll
-          for (int t = 0; t < SB; ++t) qv[t] = qn[t];
-        }
+        for (int t = 0; t < SB; ++t) qv[t] = qn[t];
       }
       __syncwarp();
 #if GBDTMO_HIST_WDEPTH == 2

@@ -24,19 +24,17 @@ __global__ void k_leaf_values(gbdtmo_problem p, const float* __restrict__ scales
 }
 
 // Leaf values from fp64 node totals summed from the leaf's rows (reading R17; the oracle's
-// definition), not from the 31-bit fixed-point sums: g, h are recomputed in fp64 from y and the
-// pre-tree prediction exactly as gbdtmo_grad computes them before quantising, so a leaf whose rows
-// all have tiny |g| (confident softmax rows: G ~ 1e-3, quantisation floor n 2^-31) is exact to fp64
-// rounding instead of to the fixed point's absolute resolution.  One block per heap node (LEAF
-// only); warp w sums a fixed contiguous part of the leaf's segment of the final row list in row
-// order, lanes over channels; the 8 warps' partials are combined in warp order: deterministic and
-// identical on every rank (replicated rows and predictions).
-constexpr int kLeafWarps = 8;
-constexpr int kLeafChunk = 256;          // channels per pass (8 fp64 accumulators per lane)
+// definition), not from the 31-bit fixed-point sums: gbdtmo_grad keeps the fp64 g, h it quantises
+// (gh), so a leaf whose rows all have tiny |g| (confident softmax rows: G ~ 1e-3 against a
+// quantisation floor of n 2^-31) is exact to fp64 rounding.  One block per heap node (LEAF only):
+// warp w sums a fixed contiguous part of the leaf's segment of the final row list in row order
+// (4 rows loaded ahead of the ordered adds), lanes over channels; the warps' partials are combined
+// in warp order: deterministic, and identical on every rank (replicated rows and gradients).
+constexpr int kLeafWarps = 32;
+constexpr int kLeafChunk = 64;           // channels per pass (2 fp64 accumulators per lane)
 
 __global__ void __launch_bounds__(kLeafWarps * 32)
-k_leaf_values_exact(gbdtmo_problem p, const float* __restrict__ y, const double* __restrict__ pred, State s,
-                    double* __restrict__ leaf) {
+k_leaf_values_exact(gbdtmo_problem p, const double* __restrict__ gh, State s, double* __restrict__ leaf) {
   extern __shared__ double lsm[];                       // [V] totals, then [kLeafWarps][kLeafChunk] partials
   const int64_t h = blockIdx.x;
   const int d = p.d, V = channels(p);
@@ -53,40 +51,28 @@ k_leaf_values_exact(gbdtmo_problem p, const float* __restrict__ y, const double*
   const int64_t per = (e - b + kLeafWarps - 1) / kLeafWarps;
   const int64_t wb = b + warp * per, we = min(e, wb + per);
   for (int c0 = 0; c0 < V; c0 += kLeafChunk) {
-    double acc[kLeafChunk / 32];
+    const int ca = c0 + lane, cb = c0 + 32 + lane;
+    const bool oa = ca < V, ob = cb < V;
+    double acc0 = 0.0, acc1 = 0.0;
+    int64_t pos = wb;
+    for (; pos + 4 <= we; pos += 4) {                   // 4 rows in flight, added in row order
+      double va[4], vb[4];
 #pragma unroll
-    for (int u = 0; u < kLeafChunk / 32; ++u) acc[u] = 0.0;
-    for (int64_t pos = wb; pos < we; ++pos) {
-      const int64_t i = rl[pos];
-      const double* pr = pred + i * d;
-      const float* yr = y + i * d;
-      double mx = -INFINITY, z = 0.0;
-      if (softmax) {                                     // p = softmax(yhat_i) (max-subtracted), R12
-        for (int k = lane; k < d; k += 32) mx = fmax(mx, pr[k]);
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-        for (int k = lane; k < d; k += 32) z += exp(pr[k] - mx);
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
+      for (int u = 0; u < 4; ++u) {
+        const double* gr = gh + (int64_t)rl[pos + u] * V;
+        va[u] = oa ? gr[ca] : 0.0;
+        vb[u] = ob ? gr[cb] : 0.0;
       }
 #pragma unroll
-      for (int u = 0; u < kLeafChunk / 32; ++u) {
-        const int c = c0 + u * 32 + lane;
-        if (c < V) {
-          double v;
-          if (!softmax) {
-            v = 2.0 * (pr[c] - (double)yr[c]);           // g = 2 (yhat - y)
-          } else {
-            const int k = c < d ? c : c - d;
-            const double pk = exp(pr[k] - mx) / z;
-            v = c < d ? pk - (double)yr[k] : pk * (1.0 - pk);   // g = p - y, h = p (1 - p)
-          }
-          acc[u] += v;
-        }
-      }
+      for (int u = 0; u < 4; ++u) { acc0 += va[u]; acc1 += vb[u]; }
     }
-#pragma unroll
-    for (int u = 0; u < kLeafChunk / 32; ++u) part[warp * kLeafChunk + u * 32 + lane] = acc[u];
+    for (; pos < we; ++pos) {
+      const double* gr = gh + (int64_t)rl[pos] * V;
+      if (oa) acc0 += gr[ca];
+      if (ob) acc1 += gr[cb];
+    }
+    part[warp * kLeafChunk + lane] = acc0;
+    part[warp * kLeafChunk + 32 + lane] = acc1;
     __syncthreads();
     for (int c = threadIdx.x; c < kLeafChunk && c0 + c < V; c += blockDim.x) {
       double t = 0.0;
@@ -153,6 +139,11 @@ __global__ void k_tree_export(gbdtmo_problem p, State s, int32_t* node_state, in
 // Without staging (rows wider than the shared-memory budget) the walk reads X from global memory.
 constexpr int kPredThreads = 512;
 
+__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(src)
+               : "memory");
+}
+
 __global__ void __launch_bounds__(kPredThreads)
 k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int T, int D, int d, int lrb, int TC,
                 int stage, const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
@@ -160,21 +151,34 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
   extern __shared__ __align__(16) unsigned char smp[];
   const int RB = 1 << lrb;
   const int mp = m | 1;
-  float* xs = reinterpret_cast<float*>(smp);
-  int16_t* lh = reinterpret_cast<int16_t*>(smp + (stage ? (size_t)RB * mp * 4 : 0));
+  float* const xs0 = reinterpret_cast<float*>(smp);
+  const int bufw = stage ? RB * mp : 0;                  // floats per staging buffer
+  int16_t* lh = reinterpret_cast<int16_t*>(smp + (stage ? (size_t)2 * RB * mp * 4 : 0));
   const int64_t NH = (int64_t(1) << (D + 1)) - 1;
   const int64_t ntiles = (n + RB - 1) >> lrb;
+  // rows of a tile are copied asynchronously (cp.async, no register round trip) one tile ahead:
+  // the next tile lands while this one is walked
+  auto stage_tile = [&](int64_t tile, float* xs) {
+    if (tile < ntiles) {
+      const int64_t r0 = tile << lrb;
+      const int rows = (int)min((int64_t)RB, n - r0);
+      for (int r = 0; r < rows; ++r) {
+        const float* src = X + (r0 + r) * ld_x;
+        float* dst = xs + r * mp;
+        for (int j = threadIdx.x; j < m; j += blockDim.x) cp_async4(dst + j, src + j);
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int buf = 0;
+  if (stage) stage_tile(blockIdx.x, xs0);
   for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int64_t r0 = tile << lrb;
     const int rows = (int)min((int64_t)RB, n - r0);
+    const float* xs = xs0 + buf * bufw;
     if (stage) {
-      for (int r = 0; r < RB; ++r) {
-        const float* src = X + (r0 + r) * ld_x;
-        float* dst = xs + r * mp;
-        if (r < rows) {
-          for (int j = threadIdx.x; j < m; j += blockDim.x) dst[j] = __ldg(&src[j]);
-        }
-      }
+      stage_tile(tile + gridDim.x, xs0 + (buf ^ 1) * bufw);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
       __syncthreads();
     }
     for (int t0 = 0; t0 < T; t0 += TC) {
@@ -216,7 +220,9 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
       }
       __syncthreads();
     }
+    buf ^= 1;
   }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
 
 __global__ void k_rows_export(gbdtmo_problem p, State s, const int32_t* __restrict__ list, int32_t* rows,
@@ -252,20 +258,19 @@ extern "C" gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx c, const gbdtmo_problem* 
 }
 
 extern "C" gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx c, const gbdtmo_problem* p, const float* scales,
-                                            void* state, const float* y, const double* pred, double* leaf) {
+                                            void* state, const double* gh, double* leaf) {
   Ctx* ctx = (Ctx*)c;
   DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
   GB_CHECK_ARG(state && leaf, "null pointer");
-  GB_CHECK_ARG((y == nullptr) == (pred == nullptr), "y and pred must be given together");
   State s = state_view(*p, state);
-  if (y) {
+  if (gh) {
     const int smem = (channels(*p) + kLeafWarps * kLeafChunk) * 8;
     static unsigned long long attr_mask = 0;
     smem_optin_once(ctx, k_leaf_values_exact, attr_mask, ctx->max_smem_optin - 1024);
-    GB_LAUNCH(k_leaf_values_exact, (unsigned)heap_nodes(*p), kLeafWarps * 32, smem, *p, y, pred, s, leaf);
+    GB_LAUNCH(k_leaf_values_exact, (unsigned)heap_nodes(*p), kLeafWarps * 32, smem, *p, gh, s, leaf);
   } else {
     GB_CHECK_ARG(scales, "null scales");
     GB_LAUNCH(k_leaf_values, 64, 256, 0, *p, scales, s, leaf);
@@ -311,16 +316,16 @@ extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n,
   GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");
   GB_CHECK_ARG(D >= 1 && D <= 12, "D out of range [1, 12]");
   if (n == 0 || T == 0) return GBDTMO_OK;
-  // rows per tile: the largest power of two <= 64 whose staged rows fit 72 KB, so 2-3 blocks share an
-  // SM and one block's staging overlaps the others' walks (0: rows too wide, read from global memory)
+  // rows per tile: the largest power of two <= 64 whose staged rows fit 36 KB (two buffers: the next
+  // tile is copied while this one is walked), 2-3 blocks per SM (0: rows too wide, read from global)
   const int64_t row_bytes = 4 * (int64_t)(m | 1);
   int lrb = 6;
-  while (lrb > 0 && (int64_t(1) << lrb) * row_bytes > 72 * 1024) --lrb;
-  const int stage = (int64_t(1) << lrb) * row_bytes <= 72 * 1024;
+  while (lrb > 0 && (int64_t(1) << lrb) * row_bytes > 36 * 1024) --lrb;
+  const int stage = (int64_t(1) << lrb) * row_bytes <= 36 * 1024;
   if (!stage) lrb = 5;
   const int RB = 1 << lrb;
   const int TC = T < 256 ? T : 256;
-  const int smem = (stage ? (int)(RB * row_bytes) : 0) + RB * TC * 2;
+  const int smem = (stage ? 2 * (int)(RB * row_bytes) : 0) + RB * TC * 2;   // two staging buffers
   static unsigned long long attr_mask = 0;
   smem_optin_once(ctx, k_predict_tiles, attr_mask, 200 * 1024);
   const int64_t ntiles = (n + RB - 1) / RB;

@@ -59,6 +59,18 @@ def _device_inputs(pkg, ctx, w):
     return ds, torch.from_numpy(Y).to(dev)
 
 
+def _first_diff(trees, ref, T):
+    """First tree whose structure differs from the oracle's (None: all equal)."""
+    for t in range(T):
+        gt = to_np(trees[t])
+        try:
+            if compare_trees(gt, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]):
+                return t
+        except AssertionError:
+            return t
+    return None
+
+
 def _check_trees(trees, ref, T, leaf_rtol=1e-5):
     for t in range(T):
         gt = to_np(trees[t])
@@ -81,8 +93,12 @@ def _check_trees(trees, ref, T, leaf_rtol=1e-5):
             np.testing.assert_allclose(gt["leaf"][leaves], ref["leaf"][t][leaves], rtol=leaf_rtol, atol=1e-7)
 
 
+# configs whose oracle is cheap enough to re-run tie-locked from the first tie on the GPU box
+TIE_LOCK = {"C2", "C3", "C4"}
+
+
 @pytest.mark.parametrize("name", ["C2", "C3", "C4", "C5"])
-def test_ten_trees_full_size_vs_oracle_golden(pkg, name):
+def test_ten_trees_full_size_vs_oracle_golden(orc, pkg, name):
     g = _golden(name)
     w = gen.WORKLOADS[name]
     T = int(g["T"])
@@ -94,6 +110,25 @@ def test_ten_trees_full_size_vs_oracle_golden(pkg, name):
     b = pkg.Booster(ctx, ds, Y, P)
     b.fit()
     torch.cuda.synchronize()
+    t0 = _first_diff(b.trees, g, T)
+    if t0 is not None:
+        # a near-tie (north star: splits may differ where gains tie within 1e-6 relative): the oracle
+        # replays trees 0..t0-1 from the golden and runs on tie-locked
+        assert name in TIE_LOCK, f"{name}: tree {t0} differs from the golden; no tie-locked re-run for this size"
+        from tests.gpu_helpers import tie_locked_oracle
+        from tools.make_golden import oracle_bins
+        _check_trees(b.trees, g, t0)
+        _, nbins, bins = oracle_bins(w)
+        X = gen.features_host(w) if w.index == 2 else None
+        y = gen.targets_host(w, X).astype(np.float64)
+        pred0 = _replay_pred(orc, bins, g, t0, w)
+        pred, ties = tie_locked_oracle(orc, bins, nbins, w.B, y, w.loss, pred0, [to_np(x) for x in b.trees], t0, T,
+                                       w.D, w.lam, w.gamma, w.lr, w.min_node)
+        print(f"{name}: ties (tree, node, gpu, oracle, rel gap): {ties}")
+        assert ties, "trees differ but no tie was found"
+        err = np.max(np.abs(b.pred.cpu().numpy() - pred))
+        assert err <= 1e-4, f"max |yhat - tie-locked oracle| after {T} trees = {err:.3e}"
+        return
     _check_trees(b.trees, g, T)
     rows = torch.from_numpy(g["sample_rows"]).cuda()
     ps = b.pred[rows].cpu().numpy()
@@ -103,6 +138,21 @@ def test_ten_trees_full_size_vs_oracle_golden(pkg, name):
     assert np.all(np.abs(s - g["pred_sum"]) <= w.n * 1e-4)
     s2 = (b.pred * b.pred).sum(0).cpu().numpy()
     assert np.all(np.abs(s2 - g["pred_sumsq"]) <= 1e-6 * np.abs(g["pred_sumsq"]) + w.n * 1e-4)
+
+
+def _replay_pred(orc, bins, g, t_end, w):
+    """yhat before tree t_end from the golden's own trees (oracle_partition + oracle_update_pred)."""
+    pred = np.zeros((w.n, w.d))
+    for t in range(t_end):
+        rows = {0: np.arange(w.n, dtype=np.int32)}
+        for h in range(g["state"].shape[1]):
+            if h not in rows:
+                continue
+            if g["state"][t][h] == 1:
+                rows[2 * h + 1], rows[2 * h + 2] = orc.partition(bins, rows[h], int(g["feat"][t][h]), int(g["bin"][t][h]))
+            elif g["state"][t][h] == 2:
+                orc.update_pred(pred, rows[h], g["leaf"][t][h])
+    return pred
 
 
 def test_ten_trees_c1_vs_oracle(orc, pkg):

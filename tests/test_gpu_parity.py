@@ -198,9 +198,10 @@ def test_grad_matches_oracle(orc, pkg, ctx, case):
     ds = pkg.bin_features(ctx, torch.from_numpy(X).to(DEV), w.B)
     b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), _params(pkg, w), pred=torch.from_numpy(pred).to(DEV))
     ctx.gbdtmo_set_stream(torch.cuda.current_stream().cuda_stream)
-    ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state)
+    ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state, b.gh)
     torch.cuda.synchronize()
     q = b.q.cpu().numpy().astype(np.float64)
+    gh = b.gh.cpu().numpy()
     sc = b.scales.cpu().numpy().astype(np.float64)
     assert np.all(np.log2(sc) == np.round(np.log2(sc)))           # powers of two
     g, h = orc.grad(w.loss, Y.astype(np.float64), pred)
@@ -214,6 +215,10 @@ def test_grad_matches_oracle(orc, pkg, ctx, case):
         hq = q[:, d:] * sc[d:]
         assert np.all(np.abs(hq - h) <= 1e-14 + sc[d:] * 0.5)
     assert np.all(np.abs(q) <= 2 ** 30)
+    # the fp64 g (and h) kept for the leaf sums: the oracle's values to fp64 rounding
+    np.testing.assert_allclose(gh[:, :d], g, rtol=1e-14, atol=1e-15)
+    if w.loss == 1:
+        np.testing.assert_allclose(gh[:, d:], h, rtol=1e-14, atol=1e-15)
 
 
 # ------------------------------------------------------------------------ histograms
@@ -358,7 +363,7 @@ def test_two_shards_equal_one(orc, pkg, ctx):
     for t in range(P.T):
         for s in shards:
             s._apply_options()
-            ctx.gbdtmo_grad(s.p, s.y, s.pred, s.q, s.scales, s.state)
+            ctx.gbdtmo_grad(s.p, s.y, s.pred, s.q, s.scales, s.state, s.gh)
         for lvl in range(P.D):
             cur, par = lvl % 2, (lvl - 1) % 2
             for s in shards:
@@ -379,7 +384,7 @@ def test_two_shards_equal_one(orc, pkg, ctx):
                 s.xchg.copy_(xs)
                 ctx.gbdtmo_partition(s.p, lvl, s.state, s.xchg)
         for s in shards:
-            ctx.gbdtmo_leaf_values(s.p, s.scales, s.state, s.leaf, s.y, s.pred)
+            ctx.gbdtmo_leaf_values(s.p, s.scales, s.state, s.leaf, s.gh)
             ctx.gbdtmo_update_pred(s.p, s.state, s.leaf, s.pred)
             s.trees.append(s.export())
     torch.cuda.synchronize()
@@ -500,10 +505,10 @@ def test_packed_bins_layout_and_equivalence(orc, pkg, ctx, case, sparse):
 
 @pytest.mark.parametrize("case", ["C2s", "C3s", "S300s"])
 def test_leaf_values_fp64_exact_vs_fixed_point(orc, pkg, ctx, case):
-    """gbdtmo_leaf_values with y / pred sums g, h in fp64 over each leaf's rows (R17): the leaves equal
+    """gbdtmo_leaf_values with gh sums g, h in fp64 over each leaf's rows (R17): the leaves equal
     the oracle's to fp64 rounding (rtol 1e-10 + 1e-13), also for confident softmax leaves whose tiny G
     sits at the fixed point's resolution floor n_leaf 2^-31 (R29); the fixed-point path
-    (y = pred = NULL) stays within that floor of them."""
+    (gh = NULL) stays within that floor of them."""
     w = CASES[case].scaled(T=4)
     X, Y = _inputs(w)
     cuts, nbins, bins = orc.bin_matrix(X, w.B)

@@ -78,7 +78,7 @@ def tree(ranks, D):
             spans.append((e0, e1))
         phases.append((name, spans))
 
-    run(lambda b: b.ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state), "grad")
+    run(lambda b: b.ctx.gbdtmo_grad(b.p, b.y, b.pred, b.q, b.scales, b.state, b.gh), "grad")
     for lvl in range(D):
         cur, par = lvl % 2, (lvl - 1) % 2
 
@@ -112,7 +112,7 @@ def tree(ranks, D):
         run(lambda b, lvl=lvl: b.ctx.gbdtmo_partition(b.p, lvl, b.state, b.xchg), f"L{lvl} partition")
 
     def fin(b):
-        b.ctx.gbdtmo_leaf_values(b.p, b.scales, b.state, b.leaf, b.y, b.pred)
+        b.ctx.gbdtmo_leaf_values(b.p, b.scales, b.state, b.leaf, b.gh)
         b.ctx.gbdtmo_update_pred(b.p, b.state, b.leaf, b.pred)
     run(fin, "leaf+update")
     return phases

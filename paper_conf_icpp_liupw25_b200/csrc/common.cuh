@@ -111,6 +111,10 @@ __host__ __device__ inline int64_t max_chunks(const gbdtmo_problem& p) {
   return p.n / kChunkMin + (int64_t(1) << p.D) + 2;
 }
 __host__ __device__ inline int64_t part_tiles(const gbdtmo_problem& p) { return (p.n + kPartTile - 1) / kPartTile; }
+constexpr int kLeafRows = 1024;        // rows per leaf-sum chunk (gbdtmo_leaf_values with fp64 g/h)
+__host__ __device__ inline int64_t leaf_chunks_max(const gbdtmo_problem& p) {
+  return p.n / kLeafRows + heap_nodes(p) + 1;
+}
 // Histogram slot of node `slot` (index within its level) in that level's buffer.  At the last
 // level (D-1 > 0) only the BUILT child of each sibling pair is ever materialised (the derived
 // one is searched as parent - built and never written), so the pair shares slot >> 1: the last
@@ -185,6 +189,7 @@ struct StateLayout {
   size_t rows0, rows1, nid;
   size_t node_begin, node_end, node_state, node_mode, node_feat, node_bin, node_gain, node_nleft, node_sum;
   size_t chunks, gnodes, snodes, misc, scale_max, tile_cnt, lpart;
+  size_t leaf_chunk, leaf_c0, leaf_part;
   size_t total;
 };
 
@@ -214,6 +219,9 @@ __host__ __device__ inline StateLayout state_layout(const gbdtmo_problem& p) {
   L.scale_max = take(8 * V);
   L.tile_cnt = take(4 * ((size_t)part_tiles(p) + 1));
   L.lpart = take(4 * NH);
+  L.leaf_chunk = take(16 * (size_t)leaf_chunks_max(p));
+  L.leaf_c0 = take(4 * (NH + 1));
+  L.leaf_part = take(8 * V * (size_t)leaf_chunks_max(p));
   L.total = o;
   return L;
 }
@@ -235,6 +243,9 @@ struct State {
   unsigned long long* scale_max;   // bits of max_i |g_ic| (fp64, non-negative)
   int32_t* tile_cnt;
   int32_t* lpart;
+  int4* leaf_chunk;   // fp64 leaf sums: (leaf, begin, end, unused) chunks of <= kLeafRows rows of the final list
+  int32_t* leaf_c0;   // [NH + 1]: first chunk of every heap node (exclusive prefix; non-leaves own none)
+  double* leaf_part;  // [chunk][V] fp64 partial sums
 };
 
 __host__ __device__ inline State state_view(const gbdtmo_problem& p, void* base) {
@@ -260,6 +271,9 @@ __host__ __device__ inline State state_view(const gbdtmo_problem& p, void* base)
   s.scale_max = (unsigned long long*)(b + L.scale_max);
   s.tile_cnt = (int32_t*)(b + L.tile_cnt);
   s.lpart = (int32_t*)(b + L.lpart);
+  s.leaf_chunk = (int4*)(b + L.leaf_chunk);
+  s.leaf_c0 = (int32_t*)(b + L.leaf_c0);
+  s.leaf_part = (double*)(b + L.leaf_part);
   return s;
 }
 

@@ -25,6 +25,7 @@
 
 #include "common.cuh"
 #include "hist_common.cuh"
+#include "tma.cuh"
 
 namespace gbdtmo {
 
@@ -66,21 +67,6 @@ HistCfg hist_config_tma(const gbdtmo_problem& p, int max_smem) {
 
 // ------------------------------------------------------------------ PTX helpers
 
-__device__ __forceinline__ void mbar_init(uint32_t addr, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(addr), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t addr, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(addr), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t addr, uint32_t parity) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n"
-      "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-      "@!p bra WAIT_%=;\n}" ::"r"(addr),
-      "r"(parity)
-      : "memory");
-}
 __device__ __forceinline__ void tma_gather4(uint32_t dst, uint64_t tmap, int col, int r0, int r1, int r2, int r3,
                                             uint32_t mbar) {
   asm volatile(

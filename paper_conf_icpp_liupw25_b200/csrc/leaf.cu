@@ -1,6 +1,7 @@
 // leaf.cu — (a)8 leaf values and (a)9 incremental prediction update,
 // plus the export of the heap-indexed tree record.
 #include "common.cuh"
+#include "plan.cuh"
 
 namespace gbdtmo {
 
@@ -26,66 +27,95 @@ __global__ void k_leaf_values(gbdtmo_problem p, const float* __restrict__ scales
 // Leaf values from fp64 node totals summed from the leaf's rows (reading R17; the oracle's
 // definition), not from the 31-bit fixed-point sums: gbdtmo_grad keeps the fp64 g, h it quantises
 // (gh), so a leaf whose rows all have tiny |g| (confident softmax rows: G ~ 1e-3 against a
-// quantisation floor of n 2^-31) is exact to fp64 rounding.  One block per heap node (LEAF only):
-// warp w sums a fixed contiguous part of the leaf's segment of the final row list in row order
-// (4 rows loaded ahead of the ordered adds), lanes over channels; the warps' partials are combined
-// in warp order: deterministic, and identical on every rank (replicated rows and gradients).
-constexpr int kLeafWarps = 32;
-constexpr int kLeafChunk = 64;           // channels per pass (2 fp64 accumulators per lane)
+// quantisation floor of n 2^-31) is exact to fp64 rounding.  Deterministic, in three steps:
+//   k_leaf_plan     every leaf's segment of the final row list is cut into chunks of <= kLeafRows
+//   k_leaf_partial  one block per chunk: warp w sums rows w, w + 8, ... in order, lanes over
+//                   channels; the 8 warps' sums are added in warp order
+//   k_leaf_final    one block per leaf: its chunks' partials added in chunk order, then Eq.
+// The order depends only on the row list, so the result is identical on every rank and run.
+constexpr int kLeafPartWarps = 8;
 
-__global__ void __launch_bounds__(kLeafWarps * 32)
-k_leaf_values_exact(gbdtmo_problem p, const double* __restrict__ gh, State s, double* __restrict__ leaf) {
-  extern __shared__ double lsm[];                       // [V] totals, then [kLeafWarps][kLeafChunk] partials
+__global__ void k_leaf_plan(gbdtmo_problem p, State s) {
+  const int64_t NH = heap_nodes(p);
+  __shared__ int sh_base;
+  if (threadIdx.x == 0) sh_base = 0;
+  __syncthreads();
+  for (int64_t h0 = 0; h0 < NH; h0 += blockDim.x) {
+    const int64_t h = h0 + threadIdx.x;
+    int nch = 0, b = 0, e = 0;
+    if (h < NH && s.node_state[h] == GBDTMO_NODE_LEAF) {
+      b = s.node_begin[h]; e = s.node_end[h];
+      nch = (e - b + kLeafRows - 1) / kLeafRows;
+    }
+    int total;
+    const int off = block_excl_scan_256(nch, &total) + sh_base;
+    if (h < NH) s.leaf_c0[h] = off;
+    for (int c = 0; c < nch; ++c) {
+      const int cb = b + c * kLeafRows;
+      s.leaf_chunk[off + c] = make_int4((int)h, cb, cb + kLeafRows < e ? cb + kLeafRows : e, 0);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) sh_base += total;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) s.leaf_c0[NH] = sh_base;
+}
+
+__global__ void __launch_bounds__(kLeafPartWarps * 32)
+k_leaf_partial(gbdtmo_problem p, const double* __restrict__ gh, State s) {
+  __shared__ double part[kLeafPartWarps][32];
+  const int64_t NH = heap_nodes(p);
+  const int V = channels(p);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int32_t* rl = (p.D & 1) ? s.rows1 : s.rows0;    // the list after the last level's partition
+  const int nchunks = s.leaf_c0[NH];
+  for (int ch = blockIdx.x; ch < nchunks; ch += gridDim.x) {
+    const int4 c4 = s.leaf_chunk[ch];
+    for (int c0 = 0; c0 < V; c0 += 32) {
+      const int c = c0 + lane;
+      double acc = 0.0;
+      int pos = c4.y + warp;
+      for (; pos + 3 * kLeafPartWarps < c4.z; pos += 4 * kLeafPartWarps) {   // 4 rows in flight, in order
+        double v[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) v[u] = c < V ? gh[(int64_t)rl[pos + u * kLeafPartWarps] * V + c] : 0.0;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc += v[u];
+      }
+      for (; pos < c4.z; pos += kLeafPartWarps)
+        if (c < V) acc += gh[(int64_t)rl[pos] * V + c];
+      part[warp][lane] = acc;
+      __syncthreads();
+      if (warp == 0 && c < V) {
+        double t = 0.0;
+#pragma unroll
+        for (int w = 0; w < kLeafPartWarps; ++w) t += part[w][lane];
+        s.leaf_part[(int64_t)ch * V + c] = t;
+      }
+      __syncthreads();
+    }
+  }
+}
+
+__global__ void k_leaf_final(gbdtmo_problem p, State s, double* __restrict__ leaf) {
   const int64_t h = blockIdx.x;
   const int d = p.d, V = channels(p);
   const bool softmax = p.loss == GBDTMO_LOSS_SOFTMAX;
-  if (s.node_state[h] != GBDTMO_NODE_LEAF) {
-    for (int k = threadIdx.x; k < d; k += blockDim.x) leaf[h * d + k] = 0.0;
-    return;
-  }
-  double* tot = lsm;
-  double* part = lsm + V;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int32_t* rl = (p.D & 1) ? s.rows1 : s.rows0;    // the list after the last level's partition
-  const int64_t b = s.node_begin[h], e = s.node_end[h];
-  const int64_t per = (e - b + kLeafWarps - 1) / kLeafWarps;
-  const int64_t wb = b + warp * per, we = min(e, wb + per);
-  for (int c0 = 0; c0 < V; c0 += kLeafChunk) {
-    const int ca = c0 + lane, cb = c0 + 32 + lane;
-    const bool oa = ca < V, ob = cb < V;
-    double acc0 = 0.0, acc1 = 0.0;
-    int64_t pos = wb;
-    for (; pos + 4 <= we; pos += 4) {                   // 4 rows in flight, added in row order
-      double va[4], vb[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const double* gr = gh + (int64_t)rl[pos + u] * V;
-        va[u] = oa ? gr[ca] : 0.0;
-        vb[u] = ob ? gr[cb] : 0.0;
-      }
-#pragma unroll
-      for (int u = 0; u < 4; ++u) { acc0 += va[u]; acc1 += vb[u]; }
-    }
-    for (; pos < we; ++pos) {
-      const double* gr = gh + (int64_t)rl[pos] * V;
-      if (oa) acc0 += gr[ca];
-      if (ob) acc1 += gr[cb];
-    }
-    part[warp * kLeafChunk + lane] = acc0;
-    part[warp * kLeafChunk + 32 + lane] = acc1;
-    __syncthreads();
-    for (int c = threadIdx.x; c < kLeafChunk && c0 + c < V; c += blockDim.x) {
-      double t = 0.0;
-      for (int w = 0; w < kLeafWarps; ++w) t += part[w * kLeafChunk + c];
-      tot[c0 + c] = t;
-    }
-    __syncthreads();
-  }
+  const bool is_leaf = s.node_state[h] == GBDTMO_NODE_LEAF;
+  const int c0 = s.leaf_c0[h], c1 = is_leaf ? s.leaf_c0[h + 1] : c0;
   const double cntd = (double)s.node_sum[h * (V + 1) + V];
   for (int k = threadIdx.x; k < d; k += blockDim.x) {
-    const double G = tot[k];
-    const double H = softmax ? tot[d + k] : 2.0 * cntd;  // MSE: h = 2 for every row
-    leaf[h * d + k] = -p.lr * G / (H + p.lambda);
+    double v = 0.0;
+    if (is_leaf) {
+      double G = 0.0, H = 0.0;
+      for (int ch = c0; ch < c1; ++ch) {
+        G += s.leaf_part[(int64_t)ch * V + k];
+        if (softmax) H += s.leaf_part[(int64_t)ch * V + d + k];
+      }
+      if (!softmax) H = 2.0 * cntd;                      // MSE: h = 2 for every row
+      v = -p.lr * G / (H + p.lambda);
+    }
+    leaf[h * d + k] = v;
   }
 }
 
@@ -138,6 +168,7 @@ __global__ void k_tree_export(gbdtmo_problem p, State s, int32_t* node_state, in
 //      bit-identical to the training prediction).
 // Without staging (rows wider than the shared-memory budget) the walk reads X from global memory.
 constexpr int kPredThreads = 512;
+constexpr int kPredW = 4;             // walks per thread in flight
 
 __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(src)
@@ -183,28 +214,48 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
     }
     for (int t0 = 0; t0 < T; t0 += TC) {
       const int tc = min(TC, T - t0);
-      for (int pq = threadIdx.x; pq < (tc << lrb); pq += blockDim.x) {
-        const int r = pq & (RB - 1), t = pq >> lrb;
-        int h = -1;
-        if (r < rows) {
-          const int64_t to = (int64_t)(t0 + t) * NH;
-          const float* xr = stage ? xs + r * mp : X + (r0 + r) * ld_x;
-          int64_t c = 0;
-          int sc = __ldg(&node_state[to]);
-          int f = __ldg(&feature[to]);
-          float th = __ldg(&threshold[to]);
-          while (sc == GBDTMO_NODE_SPLIT) {
-            if ((unsigned)f >= (unsigned)m) { sc = GBDTMO_NODE_NONE; break; }   // (malformed model)
-            const float x = stage ? xr[f] : __ldg(&xr[f]);
-            c = (x < th) ? 2 * c + 1 : 2 * c + 2;
-            if (c >= NH) { sc = GBDTMO_NODE_NONE; break; }
-            sc = __ldg(&node_state[to + c]);            // the three loads of the next node are independent
-            f = __ldg(&feature[to + c]);
-            th = __ldg(&threshold[to + c]);
+      // kPredW (row, tree) walks per thread advance level by level together: the node loads of all
+      // of them are in flight at once (memory-level parallelism for the latency-bound walk)
+      for (int pq0 = threadIdx.x; pq0 < (tc << lrb); pq0 += kPredW * blockDim.x) {
+        int64_t c[kPredW];
+        int sc[kPredW], f[kPredW], r_[kPredW], t_[kPredW];
+        float th[kPredW];
+#pragma unroll
+        for (int w = 0; w < kPredW; ++w) {
+          const int pq = pq0 + w * blockDim.x;
+          r_[w] = pq & (RB - 1);
+          t_[w] = pq >> lrb;
+          c[w] = 0;
+          sc[w] = GBDTMO_NODE_NONE;
+          if (pq < (tc << lrb) && r_[w] < rows) {
+            const int64_t to = (int64_t)(t0 + t_[w]) * NH;
+            sc[w] = __ldg(&node_state[to]);
+            f[w] = __ldg(&feature[to]);
+            th[w] = __ldg(&threshold[to]);
           }
-          h = sc == GBDTMO_NODE_LEAF ? (int)c : -1;
         }
-        lh[(r * TC) + t] = (int16_t)h;
+        for (int lv = 0; lv <= D; ++lv) {
+          bool any = false;
+#pragma unroll
+          for (int w = 0; w < kPredW; ++w) {
+            if (sc[w] != GBDTMO_NODE_SPLIT) continue;
+            if ((unsigned)f[w] >= (unsigned)m) { sc[w] = GBDTMO_NODE_NONE; continue; }   // (malformed model)
+            const float x = stage ? xs[r_[w] * mp + f[w]] : __ldg(&X[(r0 + r_[w]) * ld_x + f[w]]);
+            c[w] = (x < th[w]) ? 2 * c[w] + 1 : 2 * c[w] + 2;
+            if (c[w] >= NH) { sc[w] = GBDTMO_NODE_NONE; continue; }
+            const int64_t o = (int64_t)(t0 + t_[w]) * NH + c[w];
+            sc[w] = __ldg(&node_state[o]);
+            f[w] = __ldg(&feature[o]);
+            th[w] = __ldg(&threshold[o]);
+            any = true;
+          }
+          if (!any) break;
+        }
+#pragma unroll
+        for (int w = 0; w < kPredW; ++w) {
+          const int pq = pq0 + w * blockDim.x;
+          if (pq < (tc << lrb)) lh[(r_[w] * TC) + t_[w]] = (int16_t)(sc[w] == GBDTMO_NODE_LEAF ? (int)c[w] : -1);
+        }
       }
       __syncthreads();
       for (int e = threadIdx.x; e < rows * d; e += blockDim.x) {
@@ -267,10 +318,11 @@ extern "C" gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx c, const gbdtmo_problem* 
   GB_CHECK_ARG(state && leaf, "null pointer");
   State s = state_view(*p, state);
   if (gh) {
-    const int smem = (channels(*p) + kLeafWarps * kLeafChunk) * 8;
-    static unsigned long long attr_mask = 0;
-    smem_optin_once(ctx, k_leaf_values_exact, attr_mask, ctx->max_smem_optin - 1024);
-    GB_LAUNCH(k_leaf_values_exact, (unsigned)heap_nodes(*p), kLeafWarps * 32, smem, *p, gh, s, leaf);
+    GB_LAUNCH(k_leaf_plan, 1, kPlanThreads, 0, *p, s);
+    int64_t grid = ctx->num_sms * 8;
+    if (grid > leaf_chunks_max(*p)) grid = leaf_chunks_max(*p);
+    GB_LAUNCH(k_leaf_partial, (unsigned)grid, kLeafPartWarps * 32, 0, *p, gh, s);
+    GB_LAUNCH(k_leaf_final, (unsigned)heap_nodes(*p), 128, 0, *p, s, leaf);
   } else {
     GB_CHECK_ARG(scales, "null scales");
     GB_LAUNCH(k_leaf_values, 64, 256, 0, *p, scales, s, leaf);
@@ -316,12 +368,13 @@ extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n,
   GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");
   GB_CHECK_ARG(D >= 1 && D <= 12, "D out of range [1, 12]");
   if (n == 0 || T == 0) return GBDTMO_OK;
-  // rows per tile: the largest power of two <= 64 whose staged rows fit 36 KB (two buffers: the next
-  // tile is copied while this one is walked), 2-3 blocks per SM (0: rows too wide, read from global)
+  // rows per tile: rows of <= 1024 features are staged in shared memory (two buffers of up to 32 KB:
+  // the next tile is copied while this one is walked); wider rows are read from global memory
+  // (L1 / L2: a walk touches D of the m values) with 32-row tiles, so a tile holds 32 T walks
   const int64_t row_bytes = 4 * (int64_t)(m | 1);
   int lrb = 6;
-  while (lrb > 0 && (int64_t(1) << lrb) * row_bytes > 36 * 1024) --lrb;
-  const int stage = (int64_t(1) << lrb) * row_bytes <= 36 * 1024;
+  while (lrb > 0 && (int64_t(1) << lrb) * row_bytes > 32 * 1024) --lrb;
+  const int stage = m <= 1024 && (int64_t(1) << lrb) * row_bytes <= 32 * 1024;
   if (!stage) lrb = 5;
   const int RB = 1 << lrb;
   const int TC = T < 256 ? T : 256;

@@ -9,7 +9,6 @@
 
 #include "common.cuh"
 #include "peer.cuh"
-#include "tma.cuh"
 
 namespace gbdtmo {
 
@@ -20,9 +19,7 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_HALF
 #define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
 #endif
-#ifndef GBDTMO_FS_TMA
-#define GBDTMO_FS_TMA 1          // 1: its TMA-fed variant (k_find_split_t) where it applies
-#endif
+
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 constexpr int kRecChannels = 64; // record channels per k_split_record block
 
@@ -474,239 +471,6 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
   }
 }
 
-// TMA-fed variant of k_find_split_h (same warps, same arithmetic, bit-identical keys): the channel
-// rows a block needs -- the built child's row and, for a derived child, the parent's row, of each
-// of its features -- are streamed into a kFsStages-deep shared-memory ring by 1-D bulk copies
-// (cp.async.bulk, one elected thread, completion on an mbarrier), so the bytes in flight per SM no
-// longer depend on registers (the register-fed kernel reached 60-64% of DRAM bandwidth at 36%
-// occupancy: profiles/r01h_ncu_fs_c5.txt).  Warps read their 4 bins per row from shared memory.
-// Requires B even (16-byte rows) and 128 < B <= 256, no default bins.
-#ifndef GBDTMO_FS_STAGES
-#define GBDTMO_FS_STAGES 4
-#endif
-constexpr int kFsStages = GBDTMO_FS_STAGES;
-
-__host__ __device__ inline int fs_rows_per_stage(bool softmax, bool paired) {
-  return (softmax ? 2 : 1) * (paired ? 2 * 2 : 4);      // [g|h][feature][built|parent] or [g|h][feature (4)]
-}
-
-template <bool SOFTMAX>
-__global__ void __launch_bounds__(kFsWarps * 32, SOFTMAX ? 2 : 3)
-k_find_split_t(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
-               State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
-               const int32_t* __restrict__ pcnt, uint64_t* __restrict__ keys, int write_derived) {
-  extern __shared__ __align__(128) int64_t stg[];      // [kFsStages][rows_per_stage][B]
-  __shared__ __align__(8) unsigned long long bar_full[kFsStages], bar_empty[kFsStages];
-  __shared__ unsigned long long wbest[kFsWarps];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int half = warp & 1;
-  const bool paired = level > 0;
-  const int NF = paired ? 2 : 4, NR = paired ? 2 : 1;
-  const int fi = paired ? ((warp >> 1) & 1) : (warp >> 1);
-  const int slot = paired ? 2 * blockIdx.y + (warp >> 2) : 0;
-  const int f = (paired ? blockIdx.x * 2 : blockIdx.x * 4) + fi;
-  const int64_t first = (int64_t(1) << level) - 1;
-  const int64_t h = first + slot;
-  const int V = channels(p), B = p.B, m = p.m, d = p.d;
-  const bool searched = s.node_state[h] == GBDTMO_NODE_ACTIVE && s.node_mode[h] != MODE_SMALL;
-  const bool derive = s.node_mode[h] == MODE_DERIVE;
-  const bool store = derive && write_derived;
-  const int sib = slot ^ 1, par = slot >> 1;
-  const double lam = p.lambda;
-  const int64_t* S = s.node_sum + h * (V + 1);
-  // ---- which rows the block streams (the same set for every channel)
-  bool need_built = false, need_parent = false;
-  int64_t built_idx = 0;
-  if (paired) {
-    const int64_t hl = first + 2 * blockIdx.y, hr = hl + 1;
-    const int ml = s.node_mode[hl], mr = s.node_mode[hr];
-    const bool sl = s.node_state[hl] == GBDTMO_NODE_ACTIVE && ml != MODE_SMALL;
-    const bool sr = s.node_state[hr] == GBDTMO_NODE_ACTIVE && mr != MODE_SMALL;
-    const bool bl = ml == MODE_BUILD || ml == MODE_BUILD1, br = mr == MODE_BUILD || mr == MODE_BUILD1;
-    need_built = (bl || br) && (sl || sr);
-    need_parent = (ml == MODE_DERIVE && sl) || (mr == MODE_DERIVE && sr);
-    built_idx = hist_index(p, level, bl ? 2 * blockIdx.y : 2 * blockIdx.y + 1);
-  } else {
-    need_built = s.node_state[first] == GBDTMO_NODE_ACTIVE && s.node_mode[first] != MODE_SMALL;
-  }
-  int nfeat = min(NF, m - (int)(paired ? blockIdx.x * 2 : blockIdx.x * 4));
-  const int rows_issued = (SOFTMAX ? 2 : 1) * nfeat * ((need_built ? 1 : 0) + (need_parent ? 1 : 0));
-  const uint32_t row_bytes = (uint32_t)B * 8u;
-  const int RPS = fs_rows_per_stage(SOFTMAX, paired);
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kFsStages; ++i) {
-      mbar_init(smem_u32(&bar_full[i]), 1);
-      mbar_init(smem_u32(&bar_empty[i]), kFsWarps);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  auto issue = [&](int k) {                               // channel step k -> stage k % kFsStages
-    const int st = k % kFsStages;
-    const uint32_t fb = smem_u32(&bar_full[st]);
-    mbar_arrive_expect_tx(fb, (uint32_t)rows_issued * row_bytes);
-    int64_t* base = stg + (int64_t)st * RPS * B;
-    for (int g = 0; g < (SOFTMAX ? 2 : 1); ++g) {
-      const int ch = g == 0 ? k : d + k;
-      for (int j = 0; j < nfeat; ++j) {
-        const int fj = (paired ? blockIdx.x * 2 : blockIdx.x * 4) + j;
-        int64_t* dst = base + (int64_t)((g * NF + j) * NR) * B;
-        if (need_built) {
-          const int64_t idx = paired ? built_idx : 0;
-          bulk_g2s(smem_u32(dst), hist + ((idx * m + fj) * V + ch) * (int64_t)B, row_bytes, fb);
-        }
-        if (need_parent)
-          bulk_g2s(smem_u32(dst + B), phist + (((int64_t)blockIdx.y * m + fj) * V + ch) * (int64_t)B, row_bytes, fb);
-      }
-    }
-  };
-  if (rows_issued > 0 && threadIdx.x == 0)
-    for (int k = 0; k < min(kFsStages, d); ++k) issue(k);
-  uint64_t best = 0;
-  const int b0 = half * (32 * kFsHBins) + lane * kFsHBins;
-  const bool active = searched && f < m && half * (32 * kFsHBins) < B;
-  long long cl[kFsHBins];
-  long long ctot = 0;
-  if (active) {
-    ctot = S[V];
-    const int64_t oc = (hist_index(p, level, slot) * m + f) * B, os = (hist_index(p, level, sib) * m + f) * B,
-                  op = ((int64_t)par * m + f) * B;
-#pragma unroll
-    for (int i = 0; i < kFsHBins; ++i) {
-      const int b = b0 + i;
-      long long x = 0;
-      if (b < B) {
-        if (derive) { x = pcnt[op + b] - cnt[os + b]; if (store) cnt[oc + b] = (int32_t)x; }
-        else x = cnt[oc + b];
-      }
-      cl[i] = x;
-    }
-    half_scan(cl, half);
-    if (half) {
-#pragma unroll
-      for (int i = 0; i < kFsHBins; ++i) cl[i] = ctot - cl[i];
-    }
-  }
-  const int64_t rowc = (hist_index(p, level, slot) * m + f) * V * B;
-  double accL[kFsHBins], accR[kFsHBins];
-#pragma unroll
-  for (int i = 0; i < kFsHBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
-  double P = 0.0;
-  // a warp's own row in the stage: built row (which = 0) and parent row (which = 1) of its feature
-  auto read4 = [&](const int64_t* stage_base, int g, long long (&v)[kFsHBins], int64_t* wb) {
-    const int64_t* rb = stage_base + (int64_t)((g * NF + fi) * NR) * B;
-    if (b0 + kFsHBins <= B) {
-      const longlong2 c0 = *reinterpret_cast<const longlong2*>(rb + b0), c1 = *reinterpret_cast<const longlong2*>(rb + b0 + 2);
-      if (derive) {
-        const longlong2 a0 = *reinterpret_cast<const longlong2*>(rb + B + b0), a1 = *reinterpret_cast<const longlong2*>(rb + B + b0 + 2);
-        const longlong2 x0 = make_longlong2(a0.x - c0.x, a0.y - c0.y), x1 = make_longlong2(a1.x - c1.x, a1.y - c1.y);
-        if (wb) { reinterpret_cast<longlong2*>(wb + b0)[0] = x0; reinterpret_cast<longlong2*>(wb + b0)[1] = x1; }
-        v[0] = x0.x; v[1] = x0.y; v[2] = x1.x; v[3] = x1.y;
-      } else {
-        v[0] = c0.x; v[1] = c0.y; v[2] = c1.x; v[3] = c1.y;
-      }
-    } else {
-#pragma unroll
-      for (int i = 0; i < kFsHBins; ++i) {
-        const int b = b0 + i;
-        long long x = 0;
-        if (b < B) {
-          x = derive ? rb[B + b] - rb[b] : rb[b];
-          if (derive && wb) wb[b] = x;
-        }
-        v[i] = x;
-      }
-    }
-  };
-  for (int k = 0; k < d; ++k) {
-    const int st = k % kFsStages;
-    const uint32_t par_bit = (uint32_t)((k / kFsStages) & 1);
-    if (rows_issued > 0) mbar_wait(smem_u32(&bar_full[st]), par_bit);
-    const int64_t* sb = stg + (int64_t)st * RPS * B;
-    if (active) {
-      long long gl[kFsHBins];
-      read4(sb, 0, gl, store ? hist + rowc + (int64_t)k * B : nullptr);
-      half_scan(gl, half);
-      const long long G = S[k];
-      if (half) {
-#pragma unroll
-        for (int i = 0; i < kFsHBins; ++i) gl[i] = G - gl[i];
-      }
-      const double sg = (double)scales[k];
-      if (!SOFTMAX) {
-#pragma unroll
-        for (int i = 0; i < kFsHBins; ++i) {
-          const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
-          accL[i] = fma(GL, GL, accL[i]);
-          accR[i] = fma(GR, GR, accR[i]);
-        }
-        const double Gd = (double)G * sg;
-        P = fma(Gd, Gd, P);
-      } else {
-        long long hl[kFsHBins];
-        read4(sb, 1, hl, store ? hist + rowc + (int64_t)(d + k) * B : nullptr);
-        half_scan(hl, half);
-        const long long H = S[d + k];
-        if (half) {
-#pragma unroll
-          for (int i = 0; i < kFsHBins; ++i) hl[i] = H - hl[i];
-        }
-        const double sh = (double)scales[d + k];
-#pragma unroll
-        for (int i = 0; i < kFsHBins; ++i) {
-          const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
-          const double HL = (double)hl[i] * sh, HR = (double)(H - hl[i]) * sh;
-          accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
-        }
-        const double Gd = (double)G * sg, Hd = (double)H * sh;
-        P += Gd * Gd / (Hd + lam);
-      }
-    }
-    if (rows_issued > 0) {
-      __syncwarp();
-      if (lane == 0) mbar_arrive(smem_u32(&bar_empty[st]));
-      if (threadIdx.x == 0 && k + kFsStages < d) {       // refill this stage once every warp is done with it
-        mbar_wait(smem_u32(&bar_empty[st]), par_bit);
-        issue(k + kFsStages);
-      }
-    }
-  }
-  if (active) {
-    const int nb = nbins[f];
-    const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
-#pragma unroll
-    for (int i = 0; i < kFsHBins; ++i) {
-      const int b = b0 + i;
-      const long long c = cl[i];
-      if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
-        double gain;
-        if (!SOFTMAX)
-          gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
-                        P / (2.0 * (double)ctot + lam));
-        else
-          gain = 0.5 * (accL[i] - P);
-        if (gain > p.gamma) {
-          const uint64_t key = pack_split_key(gain, fb0 + b);
-          best = key > best ? key : best;
-        }
-      }
-    }
-  }
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
-    best = y > best ? y : best;
-  }
-  if (lane == 0) wbest[warp] = best;
-  __syncthreads();
-  if (lane == 0 && (paired ? (warp & 3) == 0 : warp == 0)) {
-    const int w0 = paired ? warp : 0, nw = paired ? kFsWarps / 2 : kFsWarps;
-    uint64_t bb = 0;
-    for (int w = w0; w < w0 + nw; ++w) bb = wbest[w] > bb ? wbest[w] : bb;
-    if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
-  }
-}
-
 __global__ void k_zero_u64(uint64_t* p, int64_t n) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = 0;
 }
@@ -912,18 +676,6 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   const int64_t LN = int64_t(1) << level;
   GB_LAUNCH(k_zero_u64, 1, 256, 0, keys, LN);
   const bool softmax = p->loss == GBDTMO_LOSS_SOFTMAX;
-  if (GBDTMO_FS_TMA && !dflt && p->B > 128 && p->B % 2 == 0) {
-    // TMA-fed half-row search: same warps and keys as k_find_split_h, channel rows streamed
-    dim3 grid(level > 0 ? (p->m + 1) / 2 : (p->m + 3) / 4, (unsigned)(level > 0 ? LN / 2 : 1));
-    const bool paired = level > 0;
-    const int smem = kFsStages * fs_rows_per_stage(softmax, paired) * p->B * 8;
-    auto kern = softmax ? k_find_split_t<true> : k_find_split_t<false>;
-    static unsigned long long attr_mask[2] = {0, 0};
-    smem_optin_once(ctx, kern, attr_mask[softmax], ctx->max_smem_optin - 1024);
-    GB_LAUNCH(kern, grid, kFsWarps * 32, smem, *p, level, nbins, scales, s, hist, cnt, level > 0 ? parent_hist : hist,
-              level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
-    return GBDTMO_OK;
-  }
   if (GBDTMO_FS_HALF && !dflt && p->B > 128) {
     // two warps per (node, feature): 2 features x 2 siblings per block, level 0: 4 features
     dim3 grid(level > 0 ? (p->m + 1) / 2 : (p->m + 3) / 4, (unsigned)(level > 0 ? LN / 2 : 1));

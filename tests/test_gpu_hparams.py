@@ -146,3 +146,14 @@ def test_near_tie_duplicate_features(orc, pkg, ctx):
         for t in range(w.T):
             assert not compare_trees(to_np(b.trees[t]), ref["state"][t], ref["feat"][t], ref["bin"][t],
                                      ref["nrows"][t]), (kw, t)
+
+
+@pytest.mark.parametrize("case,D", [("C3s", 10), ("C1", 9)])
+def test_deep_trees_vs_oracle(orc, pkg, ctx, case, D):
+    """Depth 10 (the last level keeps one histogram slot per sibling pair, R31): trees and
+    predictions equal the oracle's; min_node 5 so the deep levels really split."""
+    w = dataclasses.replace(BASE[case], D=D, T=2)
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    ref = _run(orc, pkg, ctx, w, X, Y, 1.0, 0.0, 1.0, 5, 0)
+    assert np.any(ref["state"][:, (1 << (D - 1)) - 1:(1 << D) - 1] == 1)      # splits at the last level

@@ -48,6 +48,7 @@ CASES = {
     "C4s": gen.WORKLOADS["C4"].scaled(n=20_000, m=20, T=2, D=4),
     "C5s": gen.WORKLOADS["C5"].scaled(n=50_000, m=70, T=2, D=5),
     "S300s": gen.sweep(300, n=6_000, m=24, T=2, D=3),        # NEXT-2 class sweep, d = 300 softmax
+    "S6s": gen.sweep(6, n=8_000, m=30, T=2, D=5),             # d = 6 softmax: 4 features per small-search warp
 }
 
 
@@ -288,7 +289,7 @@ def test_histograms_per_level_vs_oracle(orc, pkg, ctx, case, hk):
     ("C4s", False, 0, 0, 0), ("C5s", False, 0, 0, 0), ("S300s", False, 0, 0, 0),
     ("C3s", False, 1 << 30, 0, 0), ("C2s", True, 3000, 0, 0), ("C5s", False, 5000, 0, 0),   # global-atomic variant
     ("C1", False, 0, 2000, 0), ("C2s", False, 0, 4000, 0), ("C2s", True, 256, 2500, 0),     # sort-and-segment small nodes
-    ("C3s", False, 0, 9000, 0), ("C5s", False, 0, 6000, 0),
+    ("C3s", False, 0, 9000, 0), ("C5s", False, 0, 6000, 0), ("S6s", False, 0, 3000, 0), ("S6s", False, 0, 0, 0),
     ("C1", False, 0, 0, 1), ("C2s", False, 0, 0, 1), ("C3s", False, 0, 0, 1), ("C4s", False, 0, 0, 1),  # diagonal
     ("C5s", False, 0, 0, 1), ("S300s", False, 0, 0, 1), ("C2s", False, 3000, 128, 1),
     ("C2s", False, 0, 0, 2), ("C3s", False, 0, 0, 2), ("C4s", False, 0, 0, 2), ("C5s", False, 0, 0, 2),  # TMA-staged

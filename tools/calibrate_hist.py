@@ -21,7 +21,7 @@ import paper_conf_icpp_liupw25_b200 as pkg  # noqa: E402
 from gen import gen  # noqa: E402
 
 CANDIDATES = [0, 256, 512, 1024, 2048, 4096, 8192, 16384]
-SMALL_CANDIDATES = [0, 128, 256, 384, 512, 768, 1024]
+SMALL_CANDIDATES = [0, 128, 256, 384, 512, 768, 1024, 1536, 2048, 4096]
 
 
 def time_trees(ctx, ds, Y, w, thr, small=0, warm=2, timed=3, hk=0):

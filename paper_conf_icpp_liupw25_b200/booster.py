@@ -449,23 +449,37 @@ class Booster:
         rec["leaf"] = self.leaf.clone()
         return rec
 
-    def fit(self, T: Optional[int] = None):
-        for _ in range(T if T is not None else self.params.T):
-            self.step()
+    def fit(self, T: Optional[int] = None, graph: Optional[bool] = None):
+        """Train T trees.  graph=None: small single-process problems (n m <= 1e8, T >= 4), whose trees
+        are launch-bound (~100 launches of a few microseconds), replay trees 2.. from one captured
+        CUDA graph (identical results, tested); graph=True/False forces either."""
+        T = T if T is not None else self.params.T
+        if graph is None:
+            graph = self.group is None and T >= 4 and self.ds.n * self.ds.m <= 100_000_000
+        if graph and self.group is None and T >= 2:
+            self.step()                                  # tree 1 eagerly: allocations, attributes
+            self.capture(warmup=False)
+            for _ in range(T - 1):
+                self.step_graph()
+        else:
+            for _ in range(T):
+                self.step()
         self.check_peer(block=True)
         return self
 
     # ----------------------------------------------------------------- graphs
-    def capture(self):
-        """Capture one tree (grad .. update_pred) as a CUDA graph; replay with step_graph()."""
+    def capture(self, warmup: bool = True):
+        """Capture one tree (grad .. update_pred) as a CUDA graph; replay with step_graph().
+        warmup=False when a tree has already run eagerly on this Booster (attributes are set)."""
         s = torch.cuda.Stream(self.device)
         s.wait_stream(torch.cuda.current_stream(self.device))
-        saved = self.pred.clone()             # the warm-up tree is not part of the model
-        with torch.cuda.stream(s):
-            self._tree()                      # warm-up outside the graph (allocations, attributes)
-            self.pred.copy_(saved)
+        if warmup:
+            saved = self.pred.clone()         # the warm-up tree is not part of the model
+            with torch.cuda.stream(s):
+                self._tree()                  # warm-up outside the graph (allocations, attributes)
+                self.pred.copy_(saved)
+            del saved
         torch.cuda.current_stream(self.device).wait_stream(s)
-        del saved
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):
             self._tree()

@@ -89,6 +89,11 @@ constexpr int kPartTile = 2048;        // positions per partition block
 #endif
 constexpr int kHistThreads = GBDTMO_HIST_THREADS;   // histogram CTA (1 CTA / SM, ~200 KB smem)
 constexpr int kHistSmemBudget = 218 * 1024;   // limbs + counts + per-warp row scratch
+#ifndef GBDTMO_HIST_CTAS
+#define GBDTMO_HIST_CTAS 1        // (A/B) resident histogram CTAs per SM: 2 -> half tiles, overlapping fixed costs
+#endif
+constexpr int kHistCtas = GBDTMO_HIST_CTAS;
+constexpr int kHistTileBudget = kHistCtas == 1 ? kHistSmemBudget : (226 * 1024) / kHistCtas - 2 * 1024;
 constexpr int kHistWarps = kHistThreads / 32;
 constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte bin window)
 
@@ -163,7 +168,7 @@ __host__ __device__ inline HistCfg hist_config(const gbdtmo_problem& p) {
   for (int i = 0; i < 9; ++i) {
     const int kk = allowed[i];
     const int need = kk * limbs_per_feature + 4 * hist_cnt_words(c.K, kk, p.B) + kHistWarps * 32 * 8 * ((kk + 7) / 8);
-    if (kk <= p.m && need <= kHistSmemBudget) { k = kk; break; }
+    if (kk <= p.m && need <= kHistTileBudget) { k = kk; break; }
   }
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;

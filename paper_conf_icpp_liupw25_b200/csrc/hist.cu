@@ -47,7 +47,7 @@ __device__ __forceinline__ int dfl_of(const int (&dfl)[KF], int j) {   // dfl[j]
 }
 
 template <int K, int KF, bool SKIP, bool PACKED>
-__global__ void __launch_bounds__(kHistThreads, 1)
+__global__ void __launch_bounds__(kHistThreads, kHistCtas)
 k_hist_smem(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const uint8_t* __restrict__ packed,
             const int32_t* __restrict__ dflt, const int32_t* __restrict__ q,
             const int32_t* __restrict__ rows, int use_rows, State s,
@@ -421,7 +421,7 @@ static gbdtmo_status launch_hist_kfs(Ctx* ctx, const gbdtmo_problem& p, const Hi
                                      const int32_t* rows, int use_rows, const State& s, int64_t* hist, int32_t* cnt) {
   static unsigned long long attr_mask = 0;
   smem_optin_once(ctx, k_hist_smem<K, KF, SKIP, PACKED>, attr_mask, ctx->max_smem_optin - 1024);
-  GB_LAUNCH((k_hist_smem<K, KF, SKIP, PACKED>), ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, packed, dflt, q,
+  GB_LAUNCH((k_hist_smem<K, KF, SKIP, PACKED>), ctx->num_sms * kHistCtas, kHistThreads, hc.smem, p, hc, bins, packed, dflt, q,
             rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
 }

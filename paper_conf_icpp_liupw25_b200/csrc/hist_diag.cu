@@ -29,7 +29,7 @@ HistCfg hist_config_diag(const gbdtmo_problem& p) {
   for (int i = 0; i < 5; ++i) {
     const int kk = allowed[i];
     const int need = kk * per_feature + kHistWarps * 32 * 4 * (kk / 4 + 1);
-    if ((kk <= p.m || kk == 4) && need <= kHistSmemBudget) { k = kk; break; }
+    if ((kk <= p.m || kk == 4) && need <= kHistTileBudget) { k = kk; break; }
   }
   c.k = k;
   c.n_ft = (p.m + k - 1) / k;
@@ -60,7 +60,7 @@ struct DiagStep<S, S, R, RS, WD> {
 };
 
 template <int KF>
-__global__ void __launch_bounds__(kHistThreads, 1)
+__global__ void __launch_bounds__(kHistThreads, kHistCtas)
 k_hist_diag(gbdtmo_problem p, HistCfg hc, const uint8_t* __restrict__ bins, const int32_t* __restrict__ q,
             const int32_t* __restrict__ rows, int use_rows, State s, int64_t* __restrict__ hist,
             int32_t* __restrict__ cnt) {
@@ -231,7 +231,7 @@ static gbdtmo_status launch_diag_kf(Ctx* ctx, const gbdtmo_problem& p, const His
                                     int32_t* cnt) {
   static unsigned long long attr_mask = 0;
   smem_optin_once(ctx, k_hist_diag<KF>, attr_mask, ctx->max_smem_optin - 1024);
-  GB_LAUNCH(k_hist_diag<KF>, ctx->num_sms, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
+  GB_LAUNCH(k_hist_diag<KF>, ctx->num_sms * kHistCtas, kHistThreads, hc.smem, p, hc, bins, q, rows, use_rows, s, hist, cnt);
   return GBDTMO_OK;
 }
 

@@ -4,7 +4,7 @@
 //   hist[slot][f][c][b] = sum_{i in node, bin(i,f) = b} q[i][c],   cnt[slot][f][b] = #{...}
 // (§3.3).  What differs is how a row's bins reach the accumulating lanes.
 //
-// ncu on k_hist_smem (profiles/r01b_hist_c5_*) shows the L1 data pipe (1 wavefront / clk / SM)
+// ncu on k_hist_smem (profiles/r01h_ncu_hist_c5.txt) shows the L1 data pipe (1 wavefront / clk / SM)
 // as the limiter at 94%, and only ~60% of its wavefronts are the limb atomics that do the work:
 // each warp-wide load of 32 gathered rows' bin windows costs ~32 tag wavefronts (one per row),
 // two such loads per 32 rows, and the per-row count atomics are ~3-way bank-conflicted.  Here:

@@ -129,7 +129,8 @@ int64_t       gbdtmo_launch_count(gbdtmo_ctx ctx);
 /* ------------------------------------------------------------- size queries (host) */
 
 /* Bytes of the bins buffer: n rows of ld_bins bytes plus 32 bytes of read slack
- * (the histogram kernel loads 8-byte-aligned windows of up to 32 bytes per row). */
+ * (the histogram kernel loads 8-byte-aligned windows of up to 32 bytes per row).  Bytes past column
+ * m of a row and the slack are read but never used; zero them (once) for sanitizer-clean runs. */
 size_t gbdtmo_bins_bytes(int64_t n, int64_t ld_bins);
 /* Scratch needed by gbdtmo_bin for n rows and m columns. */
 size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B);

@@ -94,7 +94,7 @@ def bin_features(ctx: Context, X: torch.Tensor, B: int, f_begin: int = 0, m_glob
     n, m = X.shape
     ld = _align(m, 16)
     nbytes = ctx.gbdtmo_bins_bytes(n, ld)
-    bins = bins_out if bins_out is not None else torch.empty(nbytes, dtype=torch.uint8, device=X.device)
+    bins = bins_out if bins_out is not None else torch.zeros(nbytes, dtype=torch.uint8, device=X.device)
     cuts = torch.empty((m, B - 1), dtype=torch.float32, device=X.device)
     nbins = torch.empty(m, dtype=torch.int32, device=X.device)
     wsb = ctx.gbdtmo_bin_workspace_bytes(n, m, B)
@@ -136,7 +136,7 @@ def bin_features_host(ctx: Context, Xh: torch.Tensor, B: int, device, f_begin: i
     dev = torch.device(device)
     n, m = Xh.shape
     ld = _align(m, 16)
-    bins = torch.empty(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
+    bins = torch.zeros(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
     cuts = torch.empty((m, B - 1), dtype=torch.float32, device=dev)
     nbins = torch.empty(m, dtype=torch.int32, device=dev)
     sw = min(strip, m)
@@ -179,7 +179,7 @@ def bin_features_csc(ctx: Context, values: torch.Tensor, row_idx: torch.Tensor, 
     cp_dev = cp_host.to(dev)
     m = cp_host.numel() - 1
     ld = _align(m, 16)
-    bins = torch.empty(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
+    bins = torch.zeros(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
     cuts = torch.empty((m, B - 1), dtype=torch.float32, device=dev)
     nbins = torch.empty(m, dtype=torch.int32, device=dev)
     wsb = ctx.gbdtmo_bin_workspace_bytes(n, m, B)

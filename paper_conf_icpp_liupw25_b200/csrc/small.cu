@@ -183,7 +183,6 @@ k_sort_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__
     const uint16_t* sidx = reinterpret_cast<const uint16_t*>(gr + L.o_sidx);
     const unsigned char* sb = gr + L.o_sb;
     const int nb = gon ? nbins[fg] : 0;
-    const int64_t fb0 = (int64_t)(p.f_begin + (gon ? fg : 0)) * B;
     long long GL = 0, HL = 0;
     int nc = 0;                                           // candidates buffered for this lane's group
     auto flush = [&]() {

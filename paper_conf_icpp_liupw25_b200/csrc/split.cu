@@ -19,6 +19,9 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_HALF
 #define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
 #endif
+#ifndef GBDTMO_FS_PAIR
+#define GBDTMO_FS_PAIR 1         // 1: MSE channel rows loaded two at a time in k_find_split_h
+#endif
 
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 constexpr int kRecChannels = 64; // record channels per k_split_record block
@@ -347,10 +350,12 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
   uint64_t best = 0;
   const int b0 = half * (32 * kFsHBins) + lane * kFsHBins;
   if (searched && f < m && half * (32 * kFsHBins) < B) {
-    // counts -> C_L per bin
-    long long cl[kFsHBins];
-    const long long ctot = S[V];
+    // counts -> C_L per bin (kept as int32 through the channel loop: C_L < n < 2^31; this keeps
+    // the softmax instantiation inside its 80-register budget without spilling)
+    int cl[kFsHBins];
+    const int ctot = (int)S[V];
     {
+      long long cw[kFsHBins];
       const int64_t oc = (hist_index(p, level, slot) * m + f) * B, os = (hist_index(p, level, sib) * m + f) * B, op = ((int64_t)par * m + f) * B;
 #pragma unroll
       for (int i = 0; i < kFsHBins; ++i) {
@@ -360,13 +365,11 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
           if (derive) { x = pcnt[op + b] - cnt[os + b]; if (store) cnt[oc + b] = (int32_t)x; }
           else x = cnt[oc + b];
         }
-        cl[i] = x;
+        cw[i] = x;
       }
-      half_scan(cl, half);
-      if (half) {
+      half_scan(cw, half);
 #pragma unroll
-        for (int i = 0; i < kFsHBins; ++i) cl[i] = ctot - cl[i];
-      }
+      for (int i = 0; i < kFsHBins; ++i) cl[i] = (int)(half ? (long long)ctot - cw[i] : cw[i]);
     }
     const int64_t rowc = (hist_index(p, level, slot) * m + f) * V * B, rows_ = (hist_index(p, level, sib) * m + f) * V * B,
                   rowp = ((int64_t)par * m + f) * V * B;
@@ -390,15 +393,9 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
       prefetch(k);
       if (SOFTMAX) prefetch(d + k);
     }
-    for (int k = 0; k < d; ++k) {
-      if (PF > 0) {
-        prefetch(k + PF);
-        if (SOFTMAX && k + PF < d) prefetch(d + k + PF);
-      }
-      // left sums GL[i] and right sums G - GL[i] as exact integers
-      long long gl[kFsHBins];
-      load_row4(gl, b0, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
-                derive, store, B);
+    // MSE: channel rows k and k + 1 are loaded before either is scanned, so two rows' loads of each
+    // lane are in flight at once (softmax keeps one row at a time: its register budget is spent)
+    auto mse_acc = [&](long long (&gl)[kFsHBins], int k) {
       half_scan(gl, half);
       const long long G = S[k];
       if (half) {
@@ -406,16 +403,43 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
         for (int i = 0; i < kFsHBins; ++i) gl[i] = G - gl[i];
       }
       const double sg = (double)scales[k];
-      if (!SOFTMAX) {
 #pragma unroll
-        for (int i = 0; i < kFsHBins; ++i) {
-          const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
-          accL[i] = fma(GL, GL, accL[i]);
-          accR[i] = fma(GR, GR, accR[i]);
+      for (int i = 0; i < kFsHBins; ++i) {
+        const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
+        accL[i] = fma(GL, GL, accL[i]);
+        accR[i] = fma(GR, GR, accR[i]);
+      }
+      const double Gd = (double)G * sg;
+      P = fma(Gd, Gd, P);
+    };
+    for (int k = 0; k < d; k += (SOFTMAX || !GBDTMO_FS_PAIR) ? 1 : 2) {
+      if (PF > 0) {
+        prefetch(k + PF);
+        if (SOFTMAX && k + PF < d) prefetch(d + k + PF);
+        if (!SOFTMAX && GBDTMO_FS_PAIR) prefetch(k + PF + 1);
+      }
+      // left sums GL[i] and right sums G - GL[i] as exact integers
+      long long gl[kFsHBins];
+      load_row4(gl, b0, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
+                derive, store, B);
+      if (!SOFTMAX) {
+        if (GBDTMO_FS_PAIR && k + 1 < d) {
+          long long g2[kFsHBins];
+          load_row4(g2, b0, hist + rowc + (int64_t)(k + 1) * B, phist + rowp + (int64_t)(k + 1) * B,
+                    hist + rows_ + (int64_t)(k + 1) * B, derive, store, B);
+          mse_acc(gl, k);
+          mse_acc(g2, k + 1);
+        } else {
+          mse_acc(gl, k);
         }
-        const double Gd = (double)G * sg;
-        P = fma(Gd, Gd, P);
       } else {
+        half_scan(gl, half);
+        const long long G = S[k];
+        if (half) {
+#pragma unroll
+          for (int i = 0; i < kFsHBins; ++i) gl[i] = G - gl[i];
+        }
+        const double sg = (double)scales[k];
         long long hl[kFsHBins];
         load_row4(hl, b0, hist + rowc + (int64_t)(d + k) * B, phist + rowp + (int64_t)(d + k) * B,
                   hist + rows_ + (int64_t)(d + k) * B, derive, store, B);

@@ -30,6 +30,8 @@ def main():
     kw = {}
     if os.environ.get("PACKED") is not None:       # A/B: PACKED=0 row-major bins, PACKED=1 tile-packed
         kw["packed_bins"] = os.environ["PACKED"] == "1"
+    if os.environ.get("SMALL_MAX_ROWS") is not None:
+        kw["small_max_rows"] = int(os.environ["SMALL_MAX_ROWS"])
     b = pkg.Booster(ctx, ds, Y, P, **kw)
     for _ in range(trees):
         b.step()

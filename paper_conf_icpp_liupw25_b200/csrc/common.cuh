@@ -102,6 +102,17 @@ constexpr int kMaxTileFeatures = 24;   // features per histogram tile (32-byte b
 // MODE_SMALL: built from its rows and searched in shared memory (small.cu), never materialised.
 enum : int32_t { MODE_NONE = 0, MODE_BUILD = 1, MODE_DERIVE = 2, MODE_BUILD1 = 3, MODE_SMALL = 4 };
 
+// The two child terms of Eq. (3) for one output, G_L^2/(H_L + l) + G_R^2/(H_R + l), with one fp64
+// division instead of two (the softmax split search is division-bound: ncu, profiles/r02_ncu_fs_C2.txt).
+// Differs from the two-division form by a few ulp, far below the fixed-point sums' own error.
+#ifndef GBDTMO_EQ3_TWO_DIV
+#define GBDTMO_EQ3_TWO_DIV 0      // (A/B) 1: the literal two-division form
+#endif
+__device__ __forceinline__ double eq3_pair(double GL, double HLl, double GR, double HRl) {   // HLl = H_L + l, HRl = H_R + l
+  if (GBDTMO_EQ3_TWO_DIV) return GL * GL / HLl + GR * GR / HRl;
+  return fma(GL * GL, HRl, GR * GR * HLl) / (HLl * HRl);
+}
+
 // Packed split key: larger gain wins, ties -> smallest (f_global * B + b).
 __device__ __forceinline__ uint64_t pack_split_key(double gain, int64_t fb) {
   return ((uint64_t)__double_as_longlong(gain) & ~0xFFFFFFull) | (uint64_t)(0xFFFFFF - fb);

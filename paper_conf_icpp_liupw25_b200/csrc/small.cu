@@ -227,7 +227,7 @@ k_sort_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__
           const double gl = (double)GL * sg, gr_ = (double)(Gt - GL) * sg;
           double t;
           if (SOFTMAX) {
-            t = gl * gl / ((double)HL * sh + lam) + gr_ * gr_ / ((double)(Ht - HL) * sh + lam);
+            t = eq3_pair(gl, (double)HL * sh + lam, gr_, (double)(Ht - HL) * sh + lam);
           } else {
             t = gl * gl / (2.0 * (double)CL + lam) + gr_ * gr_ / (2.0 * (double)(C - CL) + lam);
           }

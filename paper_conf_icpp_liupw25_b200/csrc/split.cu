@@ -19,9 +19,7 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_HALF
 #define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
 #endif
-#ifndef GBDTMO_FS_PAIR
-#define GBDTMO_FS_PAIR 1         // 1: MSE channel rows loaded two at a time in k_find_split_h
-#endif
+
 
 constexpr int kFsBins = 8;       // bins per lane (32 x 8 = 256 = max B)
 constexpr int kRecChannels = 64; // record channels per k_split_record block
@@ -210,7 +208,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
         for (int i = 0; i < kFsBins; ++i) {
           const double GL = (double)gv[i] * sg, GR = (double)(G - gv[i]) * sg;
           const double HL = (double)hv[i] * sh, HR = (double)(H - hv[i]) * sh;
-          accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+          accL[i] += eq3_pair(GL, HL + lam, GR, HR + lam);
         }
         const double Gd = (double)G * sg, Hd = (double)H * sh;
         P += Gd * Gd / (Hd + lam);
@@ -393,8 +391,6 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
       prefetch(k);
       if (SOFTMAX) prefetch(d + k);
     }
-    // MSE: channel rows k and k + 1 are loaded before either is scanned, so two rows' loads of each
-    // lane are in flight at once (softmax keeps one row at a time: its register budget is spent)
     auto mse_acc = [&](long long (&gl)[kFsHBins], int k) {
       half_scan(gl, half);
       const long long G = S[k];
@@ -412,26 +408,17 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
       const double Gd = (double)G * sg;
       P = fma(Gd, Gd, P);
     };
-    for (int k = 0; k < d; k += (SOFTMAX || !GBDTMO_FS_PAIR) ? 1 : 2) {
+    for (int k = 0; k < d; ++k) {
       if (PF > 0) {
         prefetch(k + PF);
         if (SOFTMAX && k + PF < d) prefetch(d + k + PF);
-        if (!SOFTMAX && GBDTMO_FS_PAIR) prefetch(k + PF + 1);
       }
       // left sums GL[i] and right sums G - GL[i] as exact integers
       long long gl[kFsHBins];
       load_row4(gl, b0, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
                 derive, store, B);
       if (!SOFTMAX) {
-        if (GBDTMO_FS_PAIR && k + 1 < d) {
-          long long g2[kFsHBins];
-          load_row4(g2, b0, hist + rowc + (int64_t)(k + 1) * B, phist + rowp + (int64_t)(k + 1) * B,
-                    hist + rows_ + (int64_t)(k + 1) * B, derive, store, B);
-          mse_acc(gl, k);
-          mse_acc(g2, k + 1);
-        } else {
-          mse_acc(gl, k);
-        }
+        mse_acc(gl, k);
       } else {
         half_scan(gl, half);
         const long long G = S[k];
@@ -454,7 +441,7 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
         for (int i = 0; i < kFsHBins; ++i) {
           const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
           const double HL = (double)hl[i] * sh, HR = (double)(H - hl[i]) * sh;
-          accL[i] += GL * GL / (HL + lam) + GR * GR / (HR + lam);
+          accL[i] += eq3_pair(GL, HL + lam, GR, HR + lam);
         }
         const double Gd = (double)G * sg, Hd = (double)H * sh;
         P += Gd * Gd / (Hd + lam);

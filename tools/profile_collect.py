@@ -39,7 +39,7 @@ def launch_summary(csv_path, txt_path):
             continue
         agg[name][0] += 1
         agg[name][1] += v
-    setup = ("radix", "bin_", "k_sel_", "k_csc_", "gen_", "k_default_bins", "k_pack_bins", "at::")
+    setup = ("radix", "bin_", "k_sel_", "k_csc_", "gen_", "k_default_bins", "k_pack_bins", "at::", "k_atoms")
     tree = {k: v for k, v in agg.items() if not any(s in k for s in setup)}
     tot_tree = sum(v[1] for v in tree.values())
     with open(txt_path, "w") as f:

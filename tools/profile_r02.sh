@@ -19,6 +19,6 @@ timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
     > $out/${tag}_ncu_launches.log 2>&1
 ls -la $out/${tag}_ncu_* | head -20
 # the sort-and-segment small-node search on C2 forced to 768-row pairs (vs the histogram path)
-SMALL_MAX_ROWS=768 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_sort_search -s 2 -c 2 \
+SMALL_MAX_ROWS=768 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_sort_search -s 13 -c 3 \
    -o /tmp/${tag}_small_C2 python tools/prof_run.py C2 2 > $out/${tag}_ncu_small_C2.log 2>&1
 python tools/ncu_summary.py /tmp/${tag}_small_C2.ncu-rep --sass 25 > $out/${tag}_ncu_small_C2.txt 2>&1

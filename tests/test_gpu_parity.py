@@ -347,7 +347,7 @@ def test_partition_rows_are_stable_and_complete(orc, pkg, ctx):
 def test_two_shards_equal_one(orc, pkg, ctx):
     """Feature partitioning emulated on one GPU: two shards exchange through
     MAX(keys) and SUM(xchg) exactly as the NCCL path does; trees and predictions must equal the
-    single-shard run bit for bit."""
+    single-shard run bit for bit, and the fp64 oracle's trees (exact splits, predictions <= 1e-4)."""
     w = CASES["C3s"]
     X, Y = _inputs(w)
     Yd = torch.from_numpy(Y).to(DEV)
@@ -398,6 +398,13 @@ def test_two_shards_equal_one(orc, pkg, ctx):
             np.testing.assert_array_equal(a["leaf"], bb["leaf"])
     for s in shards:
         assert torch.equal(full.pred, s.pred)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=P.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    for t in range(P.T):
+        assert not compare_trees(to_np(shards[0].trees[t]), ref["state"][t], ref["feat"][t], ref["bin"][t],
+                                 ref["nrows"][t])
+    assert np.max(np.abs(shards[1].pred.cpu().numpy() - ref["pred"])) <= 1e-4
 
 
 def test_graph_replay_equals_eager(pkg, ctx):

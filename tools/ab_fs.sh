@@ -1,9 +1,9 @@
 #!/bin/bash
 # A/B: split search TMA-fed (default) vs register-fed half-row kernel
 mkdir -p gpurun_out
-out=gpurun_out/ab_fs_pair.jsonl; : > $out
-for wl in C5 C4 C2 S100; do
-for lib in default fs_nopair fs_sm2; do
+out=gpurun_out/ab_fs_minb4.jsonl; : > $out
+for wl in C5 C4 C3; do
+for lib in default fs_minb4; do
   if [ $lib = default ]; then L=""; else L="GBDTMO_LIB=build/ab/$lib/libgbdtmo.so"; fi
   st=10; [ $wl = C5 ] && st=8
   env $L timeout 400 python bench.py --workload $wl --no-e2e --no-cpu-baseline --steps $st --warmup 3 > gpurun_out/ab_fs_${wl}_$lib.log 2>&1

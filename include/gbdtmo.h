@@ -161,6 +161,18 @@ gbdtmo_status gbdtmo_bin(gbdtmo_ctx ctx, const float* X, int64_t n, int32_t m, i
                          uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                          void* ws, size_t ws_bytes);
 
+/* The same binning from a HOST matrix (the e2e entry point: the caller's data never needs to fit the
+ * device): X_host float32 row-major [n][ld_x] in host memory (pinned for asynchronous copies; pageable
+ * works, synchronously); the columns are uploaded in strips of `strip` columns on a copy stream owned
+ * by the context while the previous strip is binned on the context's stream (two staging buffers in
+ * ws).  bins, cuts, nbins: device, as for gbdtmo_bin.  ws: device, 256-byte aligned,
+ * gbdtmo_bin_host_workspace_bytes(n, m, B, strip) bytes.  Returns when everything is enqueued; the
+ * host matrix must stay valid until the context's stream has passed this call. */
+size_t gbdtmo_bin_host_workspace_bytes(int64_t n, int32_t m, int32_t B, int32_t strip);
+gbdtmo_status gbdtmo_bin_host(gbdtmo_ctx ctx, const float* X_host, int64_t n, int32_t m, int64_t ld_x, int32_t B,
+                              uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins, void* ws, size_t ws_bytes,
+                              int32_t strip);
+
 /* The same binning from the paper's sparse storage (Compressed Sparse Column:
  * "values", "row_indices", "col_pointers"; entries not stored are 0).  Result identical to
  * gbdtmo_bin on the dense matrix.  The implicit zeros are never materialised: they join the

@@ -28,7 +28,8 @@ SYMBOLS = (
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
     "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
     "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
-    "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async",
+    "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async", "gbdtmo_bin_host",
+    "gbdtmo_bin_host_workspace_bytes",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS = 1, 2, 3, 4
 PEER_HANDLE_BYTES = 64
@@ -76,6 +77,8 @@ def lib():
             "gbdtmo_xchg_count": ([PP, C.POINTER(i64)], C.c_int),
             "gbdtmo_bin": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz], C.c_int),
             "gbdtmo_bin_csc": ([P, P, P, P, P, i64, i32, i32, P, i64, P, P, P, sz], C.c_int),
+            "gbdtmo_bin_host": ([P, P, i64, i32, i64, i32, P, i64, P, P, P, sz, i32], C.c_int),
+            "gbdtmo_bin_host_workspace_bytes": ([i64, i32, i32, i32], sz),
             "gbdtmo_grad": ([P, PP, P, P, P, P, P, P], C.c_int),
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
@@ -192,6 +195,14 @@ class Context:
         self._check(lib().gbdtmo_bin_csc(self._h, _ptr(values), _ptr(row_idx), _ptr(col_ptr), _ptr(col_ptr_host), n,
                                          m, B, _ptr(bins), ld_bins, _ptr(cuts), _ptr(nbins), _ptr(ws), ws_bytes),
                     "gbdtmo_bin_csc")
+
+    @staticmethod
+    def gbdtmo_bin_host_workspace_bytes(n, m, B, strip) -> int:
+        return int(lib().gbdtmo_bin_host_workspace_bytes(n, m, B, strip))
+
+    def gbdtmo_bin_host(self, X_host, n, m, ld_x, B, bins, ld_bins, cuts, nbins, ws, ws_bytes, strip):
+        self._check(lib().gbdtmo_bin_host(self._h, _ptr(X_host), n, m, ld_x, B, _ptr(bins), ld_bins, _ptr(cuts),
+                                          _ptr(nbins), _ptr(ws), ws_bytes, strip), "gbdtmo_bin_host")
 
     def gbdtmo_bin(self, X, n, m, ld_x, B, bins, ld_bins, cuts, nbins, ws, ws_bytes):
         self._check(lib().gbdtmo_bin(self._h, _ptr(X), n, m, ld_x, B, _ptr(bins), ld_bins, _ptr(cuts),

@@ -110,28 +110,11 @@ def bin_features(ctx: Context, X: torch.Tensor, B: int, f_begin: int = 0, m_glob
     return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt)
 
 
-_CUDART = None
-
-
-def _memcpy2d_h2d(dst_ptr, dpitch, src_ptr, spitch, width, height, stream_handle):
-    """cudaMemcpy2DAsync host -> device (plumbing for the strip-wise upload in bin_features_host)."""
-    global _CUDART
-    import ctypes as C
-    if _CUDART is None:
-        _CUDART = C.CDLL("libcudart.so.12")
-        _CUDART.cudaMemcpy2DAsync.argtypes = [C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t, C.c_size_t, C.c_size_t,
-                                              C.c_int, C.c_void_p]
-    st = _CUDART.cudaMemcpy2DAsync(dst_ptr, dpitch, src_ptr, spitch, width, height, 1, stream_handle)
-    if st != 0:
-        raise RuntimeError(f"cudaMemcpy2DAsync failed: {st}")
-
-
 def bin_features_host(ctx: Context, Xh: torch.Tensor, B: int, device, f_begin: int = 0,
                       m_global: Optional[int] = None, strip: int = 512) -> Dataset:
-    """gbdtmo_bin on a HOST float32 matrix [n][m] (pinned for asynchronous copies), uploaded in
-    column strips on a copy stream while the previous strip is binned (binning is per column,
-    so a strip's bins, cuts and nbins are final once its call returns).  Same Dataset as
-    bin_features on the whole matrix on the device; the device never holds all of X."""
+    """gbdtmo_bin_host on a HOST float32 matrix [n][m] (pinned for asynchronous copies): the library
+    uploads it in column strips on its copy stream while the previous strip is binned (binning is per
+    column), so the device never holds all of X.  Same Dataset as bin_features on the whole matrix."""
     assert Xh.device.type == "cpu" and Xh.dtype == torch.float32 and Xh.is_contiguous()
     dev = torch.device(device)
     n, m = Xh.shape
@@ -139,32 +122,15 @@ def bin_features_host(ctx: Context, Xh: torch.Tensor, B: int, device, f_begin: i
     bins = torch.zeros(ctx.gbdtmo_bins_bytes(n, ld), dtype=torch.uint8, device=dev)
     cuts = torch.empty((m, B - 1), dtype=torch.float32, device=dev)
     nbins = torch.empty(m, dtype=torch.int32, device=dev)
-    sw = min(strip, m)
-    wsb = ctx.gbdtmo_bin_workspace_bytes(n, sw, B)
+    wsb = ctx.gbdtmo_bin_host_workspace_bytes(n, m, B, strip)
     ws = torch.empty(wsb, dtype=torch.uint8, device=dev)
-    bufs = [torch.empty((n, sw), dtype=torch.float32, device=dev) for _ in range(2)]
-    comp = torch.cuda.current_stream(dev)
-    copy = torch.cuda.Stream(dev)
-    ready = [torch.cuda.Event() for _ in range(2)]
-    free = [torch.cuda.Event() for _ in range(2)]
-    ctx.gbdtmo_set_stream(comp.cuda_stream)
-    for k, f0 in enumerate(range(0, m, sw)):
-        f1 = min(m, f0 + sw)
-        w = f1 - f0
-        j = k % 2
-        if k >= 2:
-            copy.wait_event(free[j])              # strip k-2 binned: its buffer may be refilled
-        _memcpy2d_h2d(bufs[j].data_ptr(), 4 * w, Xh.data_ptr() + 4 * f0, 4 * m, 4 * w, n, copy.cuda_stream)
-        ready[j].record(copy)
-        comp.wait_event(ready[j])
-        ctx.gbdtmo_bin(bufs[j].data_ptr(), n, w, w, B, bins.data_ptr() + f0, ld, cuts.data_ptr() + 4 * f0 * (B - 1),
-                       nbins.data_ptr() + 4 * f0, ws, wsb)
-        free[j].record(comp)
-    del bufs
+    ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
+    ctx.gbdtmo_bin_host(Xh.data_ptr(), n, m, m, B, bins, ld, cuts, nbins, ws, wsb, strip)
     dflt = torch.empty(m, dtype=torch.int32, device=dev)
     ctx.gbdtmo_default_bins(bins, n, m, ld, B, max(1, n // 16), dflt)
-    if not bool((dflt >= 0).any()):
+    if not bool((dflt >= 0).any()):          # (syncs the stream: Xh and ws are done with after this)
         dflt = None
+    del ws
     return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt)
 
 

@@ -32,7 +32,10 @@ extern "C" gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out) {
 }
 
 extern "C" gbdtmo_status gbdtmo_destroy(gbdtmo_ctx c) {
-  if (c) peer_release((Ctx*)c);
+  if (c) {
+    peer_release((Ctx*)c);
+    ctx_release_streams((Ctx*)c);
+  }
   delete (Ctx*)c;
   return GBDTMO_OK;
 }

@@ -492,9 +492,32 @@ static gbdtmo_status run_selection(Ctx* ctx, const SelWs& w, int64_t n, int tc, 
   return GBDTMO_OK;
 }
 
+void ctx_release_streams(Ctx* ctx) {
+  if (!ctx->copy_stream) return;
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(ctx->device);
+  cudaStreamSynchronize(ctx->copy_stream);
+  for (int i = 0; i < 2; ++i) {
+    if (ctx->strip_ready[i]) cudaEventDestroy(ctx->strip_ready[i]);
+    if (ctx->strip_free[i]) cudaEventDestroy(ctx->strip_free[i]);
+    ctx->strip_ready[i] = ctx->strip_free[i] = nullptr;
+  }
+  cudaStreamDestroy(ctx->copy_stream);
+  ctx->copy_stream = nullptr;
+  cudaGetLastError();
+  cudaSetDevice(prev);
+}
+
 }  // namespace gbdtmo
 
 using namespace gbdtmo;
+
+extern "C" size_t gbdtmo_bin_host_workspace_bytes(int64_t n, int32_t m, int32_t B, int32_t strip) {
+  const int64_t sw = strip < m ? strip : m;
+  const size_t stage = (size_t)(align_up((size_t)n * sw * 4, 256));
+  return 2 * stage + sel_ws_bytes(n, (int32_t)sw);
+}
 
 extern "C" size_t gbdtmo_bin_workspace_bytes(int64_t n, int32_t m, int32_t B) {
   (void)B;
@@ -526,6 +549,58 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
     GB_LAUNCH(k_bin_apply, ctx->num_sms * 2, kApplyThreads, (size_t)tc * (B - 1) * 4, X, n, ld_x, c0, tc, B, cuts,
               nbins, bins, ld_bins);
   }
+  return GBDTMO_OK;
+}
+
+extern "C" gbdtmo_status gbdtmo_bin_host(gbdtmo_ctx c, const float* X_host, int64_t n, int32_t m, int64_t ld_x,
+                                         int32_t B, uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
+                                         void* ws, size_t ws_bytes, int32_t strip) {
+  Ctx* ctx = (Ctx*)c;
+  DeviceGuard device_guard_(ctx);
+  if (!ctx) return GBDTMO_EINVAL;
+  GB_CHECK_ARG(X_host && bins && cuts && nbins && ws, "null pointer");
+  GB_CHECK_ARG(((uintptr_t)ws & 255) == 0, "ws must be 256-byte aligned");
+  GB_CHECK_ARG(n >= 1 && n < (int64_t(1) << 31) && m >= 1 && strip >= 1, "bad n, m or strip");
+  GB_CHECK_ARG(ld_x >= m && ld_bins >= m, "bad leading dimension");
+  if (B > 256) { ctx->err = "gbdtmo_bin_host: B > 256 unsupported (bins are uint8)"; return GBDTMO_EUNSUPPORTED; }
+  GB_CHECK_ARG(B >= 2, "B < 2");
+  if (ws_bytes < gbdtmo_bin_host_workspace_bytes(n, m, B, strip)) {
+    ctx->err = "gbdtmo_bin_host: workspace too small";
+    return GBDTMO_ENOMEM;
+  }
+  if (!ctx->copy_stream) {
+    if (cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking) != cudaSuccess) {
+      ctx->err = std::string("gbdtmo_bin_host: ") + cudaGetErrorString(cudaGetLastError());
+      ctx->copy_stream = nullptr;
+      return GBDTMO_ECUDA;
+    }
+    for (int i = 0; i < 2; ++i) {
+      cudaEventCreateWithFlags(&ctx->strip_ready[i], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&ctx->strip_free[i], cudaEventDisableTiming);
+    }
+  }
+  const int32_t sw = strip < m ? strip : m;
+  const size_t stage = align_up((size_t)n * sw * 4, 256);
+  float* buf[2] = {reinterpret_cast<float*>(ws), reinterpret_cast<float*>((char*)ws + stage)};
+  void* bws = (char*)ws + 2 * stage;
+  const size_t bws_bytes = ws_bytes - 2 * stage;
+  // column strips: strip k is copied (copy stream) into buf[k % 2] while strip k - 1 is binned (the
+  // context's stream); binning is per column, so a strip's bins, cuts and nbins are final
+  for (int32_t k = 0, f0 = 0; f0 < m; ++k, f0 += sw) {
+    const int32_t w = m - f0 < sw ? m - f0 : sw;
+    const int j = k & 1;
+    if (k >= 2) cudaStreamWaitEvent(ctx->copy_stream, ctx->strip_free[j], 0);   // strip k-2 binned
+    cudaMemcpy2DAsync(buf[j], (size_t)w * 4, X_host + f0, (size_t)ld_x * 4, (size_t)w * 4, (size_t)n,
+                      cudaMemcpyHostToDevice, ctx->copy_stream);
+    cudaEventRecord(ctx->strip_ready[j], ctx->copy_stream);
+    cudaStreamWaitEvent(ctx->stream, ctx->strip_ready[j], 0);
+    GB_CHECK_LAUNCH();
+    const gbdtmo_status st = gbdtmo_bin(c, buf[j], n, w, w, B, bins + f0, ld_bins, cuts + (int64_t)f0 * (B - 1),
+                                        nbins + f0, bws, bws_bytes);
+    if (st != GBDTMO_OK) return st;
+    cudaEventRecord(ctx->strip_free[j], ctx->stream);
+  }
+  GB_CHECK_LAUNCH();
   return GBDTMO_OK;
 }
 

@@ -28,8 +28,11 @@ struct Ctx {
   int64_t peer_timeout_ms = 30000;   // GBDTMO_OPT_PEER_TIMEOUT_MS: bound of every peer-flag wait
   Peer* peer = nullptr;        // gbdtmo_peer_open / _connect (peer.cu)
   const int32_t* root_cnt = nullptr;   // gbdtmo_set_root_counts: cached root counts [m][B] (or null)
+  cudaStream_t copy_stream = nullptr;  // gbdtmo_bin_host: host -> device strip copies (created on first use)
+  cudaEvent_t strip_ready[2] = {nullptr, nullptr}, strip_free[2] = {nullptr, nullptr};
   std::string err;
 };
+void ctx_release_streams(Ctx* ctx);   // bin.cu
 
 // Every entry point runs its CUDA calls on ctx->device and restores the caller's current device
 // on return (the library must not depend on, or change, the caller's current device).

@@ -634,7 +634,7 @@ def e2e_run(w, a, rank, world, local, dev, group, f0, f1, Yh, exchange="collecti
     torch.cuda.empty_cache()
     return {"value": ro / (ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": h2d // a.steps,
             "d2h_bytes_per_step": d2h // a.steps, "ms_total": ms, "trees": a.steps,
-            "what": "pkg.train(host X shard, host y): H2D + gbdtmo_bin + K trees + D2H of yhat and tree records"}
+            "what": "pkg.train(host X shard, host y): gbdtmo_bin_host (strip H2D overlapped with binning) + K trees + D2H of yhat and tree records"}
 
 
 if __name__ == "__main__":

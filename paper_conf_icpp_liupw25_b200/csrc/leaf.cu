@@ -263,7 +263,19 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
         double* pp = pred + (r0 + r) * d + k;
         double acc = *pp;
         const int16_t* hr = lh + r * TC;
-        for (int t = 0; t < tc; ++t) {
+        int t = 0;
+        for (; t + 8 <= tc; t += 8) {                    // 8 leaf loads in flight, added in tree order
+          double v[8];
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            const int h = hr[t + u];
+            v[u] = h >= 0 ? __ldg(&leaf[((int64_t)(t0 + t + u) * NH + h) * d + k]) : 0.0;
+          }
+#pragma unroll
+          for (int u = 0; u < 8; ++u)
+            if (hr[t + u] >= 0) acc += v[u];
+        }
+        for (; t < tc; ++t) {
           const int h = hr[t];
           if (h >= 0) acc += __ldg(&leaf[((int64_t)(t0 + t) * NH + h) * d + k]);
         }

@@ -319,14 +319,11 @@ __device__ __forceinline__ void load_row4(long long (&v)[kFsHBins], int b0, cons
   }
 }
 
-template <bool SOFTMAX>
-#ifndef GBDTMO_FS_HMINB
-#define GBDTMO_FS_HMINB 3        // resident blocks per SM the half-row kernel is compiled for (MSE)
-#endif
-#ifndef GBDTMO_FS_HMINB_SOFTMAX
-#define GBDTMO_FS_HMINB_SOFTMAX 3   // (4: C2 find_split 2.51 -> 2.34 ms but S500 3.0 -> 5.5 ms: spills at d = 500)
-#endif
-__global__ void __launch_bounds__(kFsWarps * 32, SOFTMAX ? GBDTMO_FS_HMINB_SOFTMAX : GBDTMO_FS_HMINB)
+// MINB = resident blocks per SM the kernel is compiled for: 3 (80 registers); MSE problems with at
+// most 16 channels take 4 (64 registers, 8 bytes spilled): C5 9.60 -> 9.27 ms per tree, while C3 / C4
+// lose 3-6% with it (profiles/r02_ab_find_split_minb4.jsonl).  Softmax keeps 3 (2: C2 2.40 -> 2.99 ms).
+template <bool SOFTMAX, int MINB>
+__global__ void __launch_bounds__(kFsWarps * 32, MINB)
 k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
                State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
                const int32_t* __restrict__ pcnt, uint64_t* __restrict__ keys, int write_derived) {
@@ -690,7 +687,8 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   if (GBDTMO_FS_HALF && !dflt && p->B > 128) {
     // two warps per (node, feature): 2 features x 2 siblings per block, level 0: 4 features
     dim3 grid(level > 0 ? (p->m + 1) / 2 : (p->m + 3) / 4, (unsigned)(level > 0 ? LN / 2 : 1));
-    auto kern = softmax ? k_find_split_h<true> : k_find_split_h<false>;
+    auto kern = softmax ? k_find_split_h<true, 3> : channels(*p) <= 16 ? k_find_split_h<false, 4>
+                                                                        : k_find_split_h<false, 3>;
     GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt, level > 0 ? parent_hist : hist,
               level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
     return GBDTMO_OK;

@@ -344,23 +344,19 @@ gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx ctx, const gbdtmo_problem* p, const 
                                  int64_t* n_rows, int64_t* n_left, const float* cuts, float* threshold);
 
 /* Inference for unseen instances ("instance-level and tree-level parallelism";
- * SURVEY NEXT-3): for every row i and tree t = 0..T-1 in order, walk from the root: at a split node
- * go left iff X[i][feature] < threshold (reading R15), at a leaf add its value:
+ * SURVEY NEXT-3): for every row i and tree t = 0..T-1 in order, walk from the root: at a SPLIT node
+ * go left iff X[i][feature] < threshold (reading R15), at a LEAF add its value:
  *   pred[i][k] += leaf[t][h][k]      (fp64, trees added in order t = 0, 1, ..., so the predictions of
  *                                     training rows equal the training path's pred bit for bit).
- * gbdtmo_pack_trees first packs the exported records (gbdtmo_tree_export: node_state / feature int32
- * [T][NH], threshold float32 [T][NH], NH = 2^(D+1)-1, 1 <= D <= 12) into nodes int32 [T][NH][2]
- * (device, 8-byte aligned, caller-owned): (feature, threshold bits) for a split, (-1, .) for a leaf,
- * (-2, .) for no node -- one 8-byte load per visited node.
- * gbdtmo_predict: X float32 row-major [n][ld_x] over ALL (global) features 0..m-1 (m <= ld_x); nodes
- * from gbdtmo_pack_trees; leaf float64 [T][NH][d] as exported; pred float64 [n][d] in/out (zeros for a
- * fresh prediction).  Rows of <= 1024 features are staged in shared memory (cp.async, double
- * buffered), wider rows are read from global memory; 4 (row, tree) walks per thread advance together.
- * A split on a feature >= m ends that walk without adding (malformed model). */
-gbdtmo_status gbdtmo_pack_trees(gbdtmo_ctx ctx, int32_t T, int32_t D, const int32_t* node_state,
-                                const int32_t* feature, const float* threshold, int32_t* nodes);
+ * X float32 row-major [n][ld_x] over ALL (global) features 0..m-1 (m <= ld_x); node_state / feature
+ * int32 [T][NH], threshold float32 [T][NH], leaf float64 [T][NH][d] as exported per tree
+ * (gbdtmo_tree_export; NH = 2^(D+1)-1, 1 <= D <= 12); pred float64 [n][d] in/out (start from zeros
+ * for a fresh prediction).  Rows are staged in shared memory in tiles (m <= ~40k features; wider
+ * rows are read from global memory); (row, tree) pairs walk concurrently.  A split on a feature
+ * >= m ends that walk without adding (malformed model). */
 gbdtmo_status gbdtmo_predict(gbdtmo_ctx ctx, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t T,
-                             int32_t D, int32_t d, const int32_t* nodes, const double* leaf, double* pred);
+                             int32_t D, int32_t d, const int32_t* node_state, const int32_t* feature,
+                             const float* threshold, const double* leaf, double* pred);
 
 /* Copy of the row bookkeeping out of `state` (tests, debugging): the row-index list as seen by
  * `level` (level = D: after the last partition), int32 [n]; the heap node of every instance,

@@ -29,7 +29,7 @@ SYMBOLS = (
     "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
     "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
     "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async", "gbdtmo_bin_host",
-    "gbdtmo_bin_host_workspace_bytes", "gbdtmo_pack_trees",
+    "gbdtmo_bin_host_workspace_bytes",
 )
 OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS = 1, 2, 3, 4
 PEER_HANDLE_BYTES = 64
@@ -92,8 +92,7 @@ def lib():
             "gbdtmo_leaf_values": ([P, PP, P, P, P, P], C.c_int),
             "gbdtmo_update_pred": ([P, PP, P, P, P], C.c_int),
             "gbdtmo_tree_export": ([P, PP, P, P, P, P, P, P, P, P, P], C.c_int),
-            "gbdtmo_predict": ([P, P, i64, i32, i64, i32, i32, i32, P, P, P], C.c_int),
-            "gbdtmo_pack_trees": ([P, i32, i32, P, P, P, P], C.c_int),
+            "gbdtmo_predict": ([P, P, i64, i32, i64, i32, i32, i32, P, P, P, P, P], C.c_int),
             "gbdtmo_rows_export": ([P, PP, P, i32, P, P, P, P], C.c_int),
             "gbdtmo_set_root_counts": ([P, P], C.c_int),
             "gbdtmo_peer_window_bytes": ([PP], sz),
@@ -267,13 +266,9 @@ class Context:
                                              _ptr(bin), _ptr(gain), _ptr(n_rows), _ptr(n_left), _ptr(cuts),
                                              _ptr(threshold)), "gbdtmo_tree_export")
 
-    def gbdtmo_pack_trees(self, T, D, node_state, feature, threshold, nodes):
-        self._check(lib().gbdtmo_pack_trees(self._h, T, D, _ptr(node_state), _ptr(feature), _ptr(threshold),
-                                            _ptr(nodes)), "gbdtmo_pack_trees")
-
-    def gbdtmo_predict(self, X, n, m, ld_x, T, D, d, nodes, leaf, pred):
-        self._check(lib().gbdtmo_predict(self._h, _ptr(X), n, m, ld_x, T, D, d, _ptr(nodes), _ptr(leaf), _ptr(pred)),
-                    "gbdtmo_predict")
+    def gbdtmo_predict(self, X, n, m, ld_x, T, D, d, node_state, feature, threshold, leaf, pred):
+        self._check(lib().gbdtmo_predict(self._h, _ptr(X), n, m, ld_x, T, D, d, _ptr(node_state), _ptr(feature),
+                                         _ptr(threshold), _ptr(leaf), _ptr(pred)), "gbdtmo_predict")
 
     def gbdtmo_rows_export(self, p, state, level, rows=None, node_of_row=None, node_begin=None, node_end=None):
         self._check(lib().gbdtmo_rows_export(self._h, C.byref(p), _ptr(state), level, _ptr(rows), _ptr(node_of_row),

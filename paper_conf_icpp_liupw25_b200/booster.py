@@ -496,7 +496,5 @@ def predict(ctx: Context, trees, X: torch.Tensor, D: int, d: int, pred: Optional
     th = torch.stack([t["threshold"] for t in trees]).contiguous()
     lf = torch.stack([t["leaf"] for t in trees]).contiguous()
     ctx.gbdtmo_set_stream(torch.cuda.current_stream(dev).cuda_stream)
-    nodes = torch.empty((T, st.shape[1], 2), dtype=torch.int32, device=dev)
-    ctx.gbdtmo_pack_trees(T, D, st, ft, th, nodes)
-    ctx.gbdtmo_predict(X, n, X.shape[1], X.stride(0), T, D, d, nodes, lf, pred)
+    ctx.gbdtmo_predict(X, n, X.shape[1], X.stride(0), T, D, d, st, ft, th, lf, pred)
     return pred

@@ -167,16 +167,6 @@ __global__ void k_tree_export(gbdtmo_problem p, State s, int32_t* node_state, in
 //      sequential order as the training path's update_pred, so predictions of training rows are
 //      bit-identical to the training prediction).
 // Without staging (rows wider than the shared-memory budget) the walk reads X from global memory.
-// Packed tree nodes for the walk: (feature, threshold bits) with feature = -1 for a leaf, -2 for no node.
-__global__ void k_pack_trees(int64_t total, const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
-                             const float* __restrict__ threshold, int2* __restrict__ nodes) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int st = node_state[i];
-    nodes[i] = make_int2(st == GBDTMO_NODE_SPLIT ? feature[i] : st == GBDTMO_NODE_LEAF ? -1 : -2,
-                         __float_as_int(threshold[i]));
-  }
-}
-
 constexpr int kPredThreads = 512;
 constexpr int kPredW = 4;             // walks per thread in flight
 
@@ -187,7 +177,8 @@ __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
 
 __global__ void __launch_bounds__(kPredThreads)
 k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int T, int D, int d, int lrb, int TC,
-                int stage, const int2* __restrict__ nodes, const double* __restrict__ leaf, double* __restrict__ pred) {
+                int stage, const int32_t* __restrict__ node_state, const int32_t* __restrict__ feature,
+                const float* __restrict__ threshold, const double* __restrict__ leaf, double* __restrict__ pred) {
   extern __shared__ __align__(16) unsigned char smp[];
   const int RB = 1 << lrb;
   const int mp = m | 1;
@@ -237,10 +228,10 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
           c[w] = 0;
           sc[w] = GBDTMO_NODE_NONE;
           if (pq < (tc << lrb) && r_[w] < rows) {
-            const int2 nd = __ldg(&nodes[(int64_t)(t0 + t_[w]) * NH]);   // one 8-byte load per node
-            f[w] = nd.x;
-            th[w] = __int_as_float(nd.y);
-            sc[w] = nd.x >= 0 ? GBDTMO_NODE_SPLIT : nd.x == -1 ? GBDTMO_NODE_LEAF : GBDTMO_NODE_NONE;
+            const int64_t to = (int64_t)(t0 + t_[w]) * NH;
+            sc[w] = __ldg(&node_state[to]);
+            f[w] = __ldg(&feature[to]);
+            th[w] = __ldg(&threshold[to]);
           }
         }
         for (int lv = 0; lv <= D; ++lv) {
@@ -252,10 +243,10 @@ k_predict_tiles(const float* __restrict__ X, int64_t n, int m, int64_t ld_x, int
             const float x = stage ? xs[r_[w] * mp + f[w]] : __ldg(&X[(r0 + r_[w]) * ld_x + f[w]]);
             c[w] = (x < th[w]) ? 2 * c[w] + 1 : 2 * c[w] + 2;
             if (c[w] >= NH) { sc[w] = GBDTMO_NODE_NONE; continue; }
-            const int2 nd = __ldg(&nodes[(int64_t)(t0 + t_[w]) * NH + c[w]]);
-            f[w] = nd.x;
-            th[w] = __int_as_float(nd.y);
-            sc[w] = nd.x >= 0 ? GBDTMO_NODE_SPLIT : nd.x == -1 ? GBDTMO_NODE_LEAF : GBDTMO_NODE_NONE;
+            const int64_t o = (int64_t)(t0 + t_[w]) * NH + c[w];
+            sc[w] = __ldg(&node_state[o]);
+            f[w] = __ldg(&feature[o]);
+            th[w] = __ldg(&threshold[o]);
             any = true;
           }
           if (!any) break;
@@ -379,28 +370,13 @@ extern "C" gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx c, const gbdtmo_problem* 
   return GBDTMO_OK;
 }
 
-extern "C" gbdtmo_status gbdtmo_pack_trees(gbdtmo_ctx c, int32_t T, int32_t D, const int32_t* node_state,
-                                           const int32_t* feature, const float* threshold, int32_t* nodes) {
-  Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
-  if (!ctx) return GBDTMO_EINVAL;
-  GB_CHECK_ARG(node_state && feature && threshold && nodes, "null pointer");
-  GB_CHECK_ARG(((uintptr_t)nodes & 7) == 0, "nodes must be 8-byte aligned");
-  GB_CHECK_ARG(T >= 0 && D >= 1 && D <= 12, "bad shape");
-  const int64_t total = (int64_t)T * ((int64_t(1) << (D + 1)) - 1);
-  if (total == 0) return GBDTMO_OK;
-  GB_LAUNCH(k_pack_trees, ctx->num_sms * 2, 256, 0, total, node_state, feature, threshold,
-            reinterpret_cast<int2*>(nodes));
-  return GBDTMO_OK;
-}
-
 extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n, int32_t m, int64_t ld_x, int32_t T,
-                                        int32_t D, int32_t d, const int32_t* nodes, const double* leaf, double* pred) {
+                                        int32_t D, int32_t d, const int32_t* node_state, const int32_t* feature,
+                                        const float* threshold, const double* leaf, double* pred) {
   Ctx* ctx = (Ctx*)c;
   DeviceGuard device_guard_(ctx);
   if (!ctx) return GBDTMO_EINVAL;
-  GB_CHECK_ARG(X && nodes && leaf && pred, "null pointer");
-  GB_CHECK_ARG(((uintptr_t)nodes & 7) == 0, "nodes must be 8-byte aligned");
+  GB_CHECK_ARG(X && node_state && feature && threshold && leaf && pred, "null pointer");
   GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");
   GB_CHECK_ARG(D >= 1 && D <= 12, "D out of range [1, 12]");
   if (n == 0 || T == 0) return GBDTMO_OK;
@@ -422,7 +398,7 @@ extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n,
   per_sm = per_sm < 1 ? 1 : per_sm > 4 ? 4 : per_sm;
   int64_t grid = (int64_t)ctx->num_sms * per_sm;
   if (grid > ntiles) grid = ntiles;
-  GB_LAUNCH(k_predict_tiles, (unsigned)grid, kPredThreads, smem, X, n, m, ld_x, T, D, d, lrb, TC, stage,
-            reinterpret_cast<const int2*>(nodes), leaf, pred);
+  GB_LAUNCH(k_predict_tiles, (unsigned)grid, kPredThreads, smem, X, n, m, ld_x, T, D, d, lrb, TC, stage, node_state,
+            feature, threshold, leaf, pred);
   return GBDTMO_OK;
 }

@@ -158,7 +158,10 @@ int target_chunks_for(const Ctx* ctx, const gbdtmo_problem& p) {
                : (ctx->hist_kernel == 2 && hist_tma_supported(p, nullptr)) ? hist_config_tma(p, ctx->max_smem_optin)
                                                                           : hist_config(p);
   int64_t tiles = (int64_t)hc.n_ft * hc.n_ct;
-  int64_t want = 4LL * ctx->num_sms * kHistCtas;
+#ifndef GBDTMO_HIST_WAVES
+#define GBDTMO_HIST_WAVES 4   // work items wanted per level, in multiples of the SM count
+#endif
+  int64_t want = (int64_t)GBDTMO_HIST_WAVES * ctx->num_sms * kHistCtas;
   int64_t t = (want + tiles - 1) / tiles;
   return (int)(t < 1 ? 1 : t);
 }

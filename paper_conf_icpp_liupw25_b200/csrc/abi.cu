@@ -19,7 +19,7 @@ extern "C" gbdtmo_status gbdtmo_create(int device, gbdtmo_ctx* out) {
   Ctx* ctx = new (std::nothrow) Ctx();
   if (!ctx) return GBDTMO_ENOMEM;
   ctx->device = device;
-  DeviceGuard device_guard_(ctx);          // restores the caller's device on return
+  GB_ENTRY(ctx);          // restores the caller's device on return
   if (cudaGetLastError() != cudaSuccess ||
       cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
       cudaDeviceGetAttribute(&ctx->max_smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device) != cudaSuccess) {
@@ -42,7 +42,7 @@ extern "C" gbdtmo_status gbdtmo_destroy(gbdtmo_ctx c) {
 
 extern "C" gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx c, void* stream) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   ctx->stream = (cudaStream_t)stream;
   return GBDTMO_OK;
@@ -50,7 +50,7 @@ extern "C" gbdtmo_status gbdtmo_set_stream(gbdtmo_ctx c, void* stream) {
 
 extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t value) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   switch (option) {
     case GBDTMO_OPT_GMEM_MAX_ROWS: ctx->gmem_max_rows = value; return GBDTMO_OK;
@@ -69,13 +69,13 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
 
 extern "C" const char* gbdtmo_last_error(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   return ctx ? ctx->err.c_str() : "null context";
 }
 
 extern "C" int64_t gbdtmo_launch_count(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   return ctx ? ctx->launches : -1;
 }
 

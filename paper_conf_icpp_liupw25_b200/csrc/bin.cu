@@ -528,7 +528,7 @@ extern "C" gbdtmo_status gbdtmo_bin(gbdtmo_ctx c, const float* X, int64_t n, int
                                     uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins, void* ws,
                                     size_t ws_bytes) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X && bins && cuts && nbins && ws, "null pointer");
   GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
@@ -556,7 +556,7 @@ extern "C" gbdtmo_status gbdtmo_bin_host(gbdtmo_ctx c, const float* X_host, int6
                                          int32_t B, uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                                          void* ws, size_t ws_bytes, int32_t strip) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X_host && bins && cuts && nbins && ws, "null pointer");
   GB_CHECK_ARG(((uintptr_t)ws & 255) == 0, "ws must be 256-byte aligned");
@@ -609,7 +609,7 @@ extern "C" gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx c, const float* values, const
                                         int32_t B, uint8_t* bins, int64_t ld_bins, float* cuts, int32_t* nbins,
                                         void* ws, size_t ws_bytes) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(col_ptr && col_ptr_host && bins && cuts && nbins && ws, "null pointer");
   GB_CHECK_ARG(((uintptr_t)ws & 15) == 0, "ws must be 16-byte aligned");
@@ -645,7 +645,7 @@ extern "C" gbdtmo_status gbdtmo_bin_csc(gbdtmo_ctx c, const float* values, const
 extern "C" gbdtmo_status gbdtmo_default_bins(gbdtmo_ctx c, const uint8_t* bins, int64_t n, int32_t m, int64_t ld_bins,
                                              int32_t B, int64_t min_count, int32_t* dflt) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(bins && dflt, "null pointer");
   GB_CHECK_ARG(n >= 1 && m >= 1 && ld_bins >= m && ld_bins % 8 == 0 && B >= 2 && B <= 256, "bad shape");

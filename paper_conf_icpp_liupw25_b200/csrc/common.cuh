@@ -2,6 +2,7 @@
 // of libgbdtmo.so (the product path).  Nothing here is shared with oracle/.
 #pragma once
 
+#include <nvtx3/nvToolsExt.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdio.h>
@@ -49,6 +50,18 @@ struct DeviceGuard {
     if (prev >= 0) cudaSetDevice(prev);
   }
 };
+
+// NVTX range over one C-ABI call (tracing): shows every entry point by name in Nsight
+// Systems and `ncu --nvtx` filters; a no-op branch unless a tool is attached (header-only NVTX3).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+// Every extern "C" entry point opens with GB_ENTRY(ctx): the context's device made current (the
+// caller's restored on return) and an NVTX range named after the call.
+#define GB_ENTRY(ctx)               \
+  DeviceGuard device_guard_(ctx);   \
+  NvtxRange nvtx_range_(__func__)
 
 // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) applies per device: one bit per device per
 // kernel instantiation (the caller keeps a static mask), set with the context's device current.

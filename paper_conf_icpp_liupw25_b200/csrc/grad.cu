@@ -173,7 +173,7 @@ using namespace gbdtmo;
 extern "C" gbdtmo_status gbdtmo_grad(gbdtmo_ctx c, const gbdtmo_problem* p, const float* y, const double* pred,
                                      int32_t* q, float* scales, void* state, double* gh) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");

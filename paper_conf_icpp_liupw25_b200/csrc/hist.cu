@@ -516,7 +516,7 @@ extern "C" gbdtmo_status gbdtmo_build_hist(gbdtmo_ctx c, const gbdtmo_problem* p
                                            const uint8_t* bins, const int32_t* dflt, const int32_t* q, void* state,
                                            int64_t* hist, int32_t* cnt) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -530,7 +530,7 @@ extern "C" gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx c, const gbdtmo_pro
                                                   const uint8_t* bins, const uint8_t* packed, const int32_t* dflt,
                                                   const int32_t* q, void* state, int64_t* hist, int32_t* cnt) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -550,7 +550,7 @@ extern "C" size_t gbdtmo_packed_bins_bytes(const gbdtmo_problem* p) {
 extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p, const uint8_t* bins,
                                           uint8_t* packed) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -564,7 +564,7 @@ extern "C" gbdtmo_status gbdtmo_pack_bins(gbdtmo_ctx c, const gbdtmo_problem* p,
 
 extern "C" gbdtmo_status gbdtmo_set_root_counts(gbdtmo_ctx c, const int32_t* root_cnt) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   ctx->root_cnt = root_cnt;
   return GBDTMO_OK;

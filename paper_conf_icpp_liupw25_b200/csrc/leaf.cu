@@ -309,7 +309,7 @@ extern "C" gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx c, const gbdtmo_problem* 
                                             int32_t* rows, int32_t* node_of_row, int32_t* node_begin,
                                             int32_t* node_end) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -323,7 +323,7 @@ extern "C" gbdtmo_status gbdtmo_rows_export(gbdtmo_ctx c, const gbdtmo_problem* 
 extern "C" gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx c, const gbdtmo_problem* p, const float* scales,
                                             void* state, const double* gh, double* leaf) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -345,7 +345,7 @@ extern "C" gbdtmo_status gbdtmo_leaf_values(gbdtmo_ctx c, const gbdtmo_problem* 
 extern "C" gbdtmo_status gbdtmo_update_pred(gbdtmo_ctx c, const gbdtmo_problem* p, const void* state,
                                             const double* leaf, double* pred) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -359,7 +359,7 @@ extern "C" gbdtmo_status gbdtmo_tree_export(gbdtmo_ctx c, const gbdtmo_problem* 
                                             int32_t* node_state, int32_t* feature, int32_t* bin, double* gain,
                                             int64_t* n_rows, int64_t* n_left, const float* cuts, float* threshold) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -374,7 +374,7 @@ extern "C" gbdtmo_status gbdtmo_predict(gbdtmo_ctx c, const float* X, int64_t n,
                                         int32_t D, int32_t d, const int32_t* node_state, const int32_t* feature,
                                         const float* threshold, const double* leaf, double* pred) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(X && node_state && feature && threshold && leaf && pred, "null pointer");
   GB_CHECK_ARG(n >= 0 && T >= 0 && m >= 1 && ld_x >= m && d >= 1, "bad shape");

@@ -225,7 +225,7 @@ static gbdtmo_status partition_impl(Ctx* ctx, const gbdtmo_problem* p, int32_t l
 extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, void* state,
                                           const int64_t* xchg) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -237,7 +237,7 @@ extern "C" gbdtmo_status gbdtmo_partition(gbdtmo_ctx c, const gbdtmo_problem* p,
 extern "C" gbdtmo_status gbdtmo_partition_peer(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, void* state,
                                                int64_t* xchg_merged) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");

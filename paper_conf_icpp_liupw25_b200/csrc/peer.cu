@@ -109,7 +109,7 @@ extern "C" size_t gbdtmo_peer_window_bytes(const gbdtmo_problem* p) {
 extern "C" gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t rank, int32_t world,
                                           uint8_t* handle) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -140,7 +140,7 @@ extern "C" gbdtmo_status gbdtmo_peer_open(gbdtmo_ctx c, const gbdtmo_problem* p,
 
 extern "C" gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx c, const uint8_t* handles) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(ctx->peer, "gbdtmo_peer_open first");
   GB_CHECK_ARG(handles, "null handles");
@@ -167,7 +167,7 @@ extern "C" gbdtmo_status gbdtmo_peer_connect(gbdtmo_ctx c, const uint8_t* handle
 extern "C" gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx c, const gbdtmo_problem* p, int32_t level, uint64_t** keys,
                                              int64_t** xchg) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -180,7 +180,7 @@ extern "C" gbdtmo_status gbdtmo_peer_buffers(gbdtmo_ctx c, const gbdtmo_problem*
 
 extern "C" gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx c, int64_t* epoch, int64_t* error) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(ctx->peer, "no peer window");
   uint64_t hdr[PEER_HEADER_WORDS];
@@ -195,7 +195,7 @@ extern "C" gbdtmo_status gbdtmo_peer_status(gbdtmo_ctx c, int64_t* epoch, int64_
 
 extern "C" gbdtmo_status gbdtmo_peer_status_async(gbdtmo_ctx c, int64_t* out) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   GB_CHECK_ARG(ctx->peer, "no peer window");
   GB_CHECK_ARG(out, "null output");
@@ -210,7 +210,7 @@ extern "C" gbdtmo_status gbdtmo_peer_status_async(gbdtmo_ctx c, int64_t* out) {
 
 extern "C" gbdtmo_status gbdtmo_peer_close(gbdtmo_ctx c) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   peer_release(ctx);
   return GBDTMO_OK;

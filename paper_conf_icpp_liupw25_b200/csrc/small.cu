@@ -266,7 +266,7 @@ extern "C" gbdtmo_status gbdtmo_search_small(gbdtmo_ctx c, const gbdtmo_problem*
                                              const uint8_t* bins, const int32_t* q, const int32_t* nbins,
                                              const float* scales, void* state, uint64_t* keys) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");

@@ -673,7 +673,7 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
                                            int64_t* hist, int32_t* cnt, const int64_t* parent_hist,
                                            const int32_t* parent_cnt, uint64_t* keys) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -727,7 +727,7 @@ extern "C" gbdtmo_status gbdtmo_split_record(gbdtmo_ctx c, const gbdtmo_problem*
                                              const int64_t* parent_hist, const int32_t* parent_cnt,
                                              const uint64_t* keys, int64_t* xchg) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");
@@ -747,7 +747,7 @@ extern "C" gbdtmo_status gbdtmo_split_record_peer(gbdtmo_ctx c, const gbdtmo_pro
                                                   const int64_t* parent_hist, const int32_t* parent_cnt,
                                                   uint64_t* keys_merged) {
   Ctx* ctx = (Ctx*)c;
-  DeviceGuard device_guard_(ctx);
+  GB_ENTRY(ctx);
   if (!ctx) return GBDTMO_EINVAL;
   const char* bad = check_problem(p);
   GB_CHECK_ARG(!bad, bad ? bad : "");

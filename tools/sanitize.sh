@@ -16,7 +16,7 @@ run() {   # tool case variant
 }
 for tool in memcheck racecheck synccheck; do
   for v in k0 k1 k2 gmem small; do run $tool C1 $v; run $tool C3s $v; done
-  run $tool C2s k1; run $tool C2s sparse; run $tool C2s small; run $tool C1 graph; run $tool C3s predict
+  run $tool C2s k1; run $tool C2s sparse; run $tool C2s small; run $tool C1 graph; run $tool C3s predict; run $tool C3s binhost; run $tool C3s packed
 done
 # initcheck on the default path (uninitialised device reads)
 run initcheck C3s k0; run initcheck C2s k1

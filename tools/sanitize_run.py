@@ -3,8 +3,9 @@
   python tools/sanitize_run.py <case> <variant>
 case: C1 | C3s | C2s;  variant: k0 (row-pair smem), k1 (diagonal), k2 (TMA-staged), gmem (global
 atomics for every node), small (sort-and-segment small nodes), sparse (default-bin skip), graph
-(CUDA-graph replay), predict (gbdtmo_predict).  Prints the max |pred - oracle| (parity still holds
-under the tool)."""
+(CUDA-graph replay), predict (gbdtmo_predict), binhost (train() from a pinned host matrix:
+gbdtmo_bin_host strip uploads on the context's copy stream), packed (tile-packed bins).  Prints
+the max |pred - oracle| (parity still holds under the tool)."""
 import os
 import sys
 
@@ -35,10 +36,16 @@ def main():
               gmem=dict(gmem_max_rows=1 << 30, small_max_rows=0),
               small=dict(small_max_rows=4000, gmem_max_rows=0),
               sparse=dict(sparse_default=True, hist_kernel=0),
-              graph=dict(), predict=dict())[var]
+              graph=dict(), predict=dict(), binhost=dict(), packed=dict(packed_bins=True, hist_kernel=0))[var]
     P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
-    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P, **kw)
-    if var == "graph":
+    if var == "binhost":
+        b = pkg.train(torch.from_numpy(X).pin_memory(), torch.from_numpy(Y), P, ctx=ctx)
+    else:
+        b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P,
+                        **kw)
+    if var == "binhost":
+        pass
+    elif var == "graph":
         b.capture()
         for _ in range(w.T):
             b.step_graph()

@@ -111,9 +111,16 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *     instruction each adding to a different slot, conflict-free for any channel count (DESIGN.md
  *     §7); 2: row-pair tiles whose bin windows are staged in shared memory by TMA gather4
  *     (measured slower, kept as the recorded alternative).  Same results; chosen per workload
- *     shape by measurement.  1 and 2 are not used with default bins. */
+ *     shape by measurement.  1 and 2 are not used with default bins.
+ *   GBDTMO_OPT_FS_CHANNEL_GROUPS: split search parallelism (gbdtmo_find_split, B > 128, no default
+ *     bins) — 0 (default): automatic: a level whose (node, feature) warps would not fill the GPU
+ *     (fewer than 32 / CG warps per SM) splits every (node, feature)'s channel loop over CG = 2, 4
+ *     or 8 warp pairs whose Eq. (3) partial sums are added in shared memory in a fixed order; 1:
+ *     never; 2 / 4 / 8: always, with that CG (at most d).  Same (f, b) decisions up to near-ties;
+ *     gains differ by fp64 summation order. */
 enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3,
-       GBDTMO_OPT_PEER_TIMEOUT_MS = 4 /* bound of every peer-flag wait (gbdtmo_peer_*), default 30000 */ };
+       GBDTMO_OPT_PEER_TIMEOUT_MS = 4 /* bound of every peer-flag wait (gbdtmo_peer_*), default 30000 */,
+       GBDTMO_OPT_FS_CHANNEL_GROUPS = 5 };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Cached root counts.  The root holds all n rows in every tree, so its count histogram
  * cnt[0][f][b] = #{i : bin(i, f) = b} (PAPER.md:214's histogram, count channel) is the same for

@@ -167,10 +167,12 @@ class Booster:
                  group=None, pred: Optional[torch.Tensor] = None, keep_model: bool = True,
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
                  small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
-                 packed_bins: Optional[bool] = None, exchange: str = "collective", cache_root_counts: bool = True):
+                 packed_bins: Optional[bool] = None, exchange: str = "collective", cache_root_counts: bool = True,
+                 fs_channel_groups: int = 0):
         """exchange (only with `group`): "collective" = torch.distributed all-reduces per level;
         "peer" = the fused peer-memory exchange (NEXT-4, gbdtmo_*_peer): the keys / records are
-        read from the other ranks' windows inside split_record / partition, no host collective."""
+        read from the other ranks' windows inside split_record / partition, no host collective.
+        fs_channel_groups: GBDTMO_OPT_FS_CHANNEL_GROUPS (0 automatic, 1 off, 2 / 4 / 8 forced)."""
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
         assert exchange in ("collective", "peer")
         self.exchange = exchange if group is not None else "collective"
@@ -186,6 +188,7 @@ class Booster:
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
+        self.fs_channel_groups = int(fs_channel_groups)
         dev = ds.bins.device
         self.device = dev
         n, d = y.shape
@@ -353,6 +356,7 @@ class Booster:
         ctx.gbdtmo_set_option(_abi.OPT_GMEM_MAX_ROWS, self.gmem_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_HIST_KERNEL, self.hist_kernel)
+        ctx.gbdtmo_set_option(_abi.OPT_FS_CHANNEL_GROUPS, self.fs_channel_groups)
         ctx.gbdtmo_set_root_counts(self.root_cnt)
 
     def _mark(self, name: str, on: bool):

@@ -63,6 +63,13 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
       if (value < 1) { ctx->err = "gbdtmo_set_option: PEER_TIMEOUT_MS must be >= 1"; return GBDTMO_EINVAL; }
       ctx->peer_timeout_ms = value;
       return GBDTMO_OK;
+    case GBDTMO_OPT_FS_CHANNEL_GROUPS:
+      if (value != 0 && value != 1 && value != 2 && value != 4 && value != 8) {
+        ctx->err = "gbdtmo_set_option: FS_CHANNEL_GROUPS must be 0, 1, 2, 4 or 8";
+        return GBDTMO_EINVAL;
+      }
+      ctx->fs_channel_groups = value;
+      return GBDTMO_OK;
     default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;
   }
 }

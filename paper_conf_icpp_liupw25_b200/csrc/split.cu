@@ -16,6 +16,9 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_PF
 #define GBDTMO_FS_PF 2           // channels of L2 prefetch ahead in the split search
 #endif
+#ifndef GBDTMO_FS_CG_OFF
+#define GBDTMO_FS_CG_OFF 0       // (A/B) 1: no channel-split search (k_find_split_c)
+#endif
 #ifndef GBDTMO_FS_HALF
 #define GBDTMO_FS_HALF 1         // 1: half-row split search (k_find_split_h) where it applies
 #endif
@@ -479,6 +482,175 @@ k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, c
   }
 }
 
+// Channel-split search for shallow levels of wide problems: the half-row kernel
+// gives every (node, feature) two warps that each walk all V channel rows, so a level with few
+// nodes x features leaves most SMs idle (C4 root: 125 blocks for 148 SMs, 12% occupancy, 22% of
+// HBM; C3 root: 25 blocks).  Eq. (3) is a sum over outputs, so the channel loop splits: one block
+// per (node, feature), warps = [channel group cg < CG][half]; warp (cg, half) takes outputs
+// k = cg, cg + CG, ... of its half's bins, and the per-bin partial sums (sum_k G_L^2, sum_k G_R^2,
+// sum_k G^2 for MSE; the Eq. (3) terms for softmax) are added in shared memory in cg order (a fixed
+// order: deterministic; the sums differ from the sequential kernel's by fp64 rounding only).
+// Integer work (prefix sums, derived rows, validity) is exactly k_find_split_h's.
+// Blocks are (slot, feature) with the slot fastest, so the two children of a split run side by
+// side and the derived child's reads of its built sibling hit L2.
+template <bool SOFTMAX, int CGMAX>
+__global__ void __launch_bounds__(2 * 32 * CGMAX, CGMAX <= 4 ? 3 : 1)
+k_find_split_c(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
+               State s, int64_t* __restrict__ hist, int32_t* __restrict__ cnt, const int64_t* __restrict__ phist,
+               const int32_t* __restrict__ pcnt, uint64_t* __restrict__ keys, int write_derived) {
+  constexpr int kFsCgMax = CGMAX;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int half = warp & 1, cg = warp >> 1, CG = blockDim.x >> 6;
+  const int slot = blockIdx.x, f = blockIdx.y;
+  const int64_t h = (int64_t(1) << level) - 1 + slot;
+  // block-uniform exits (before any barrier)
+  if (!(s.node_state[h] == GBDTMO_NODE_ACTIVE && s.node_mode[h] != MODE_SMALL) || f >= p.m) return;
+  const bool derive = level > 0 && s.node_mode[h] == MODE_DERIVE;
+  const bool store = derive && write_derived;
+  const int V = channels(p), B = p.B, m = p.m, d = p.d;
+  const int sib = slot ^ 1, par = slot >> 1;
+  const double lam = p.lambda;
+  const int64_t* S = s.node_sum + h * (V + 1);
+  constexpr int NP = 2 * kFsHBins + 1;                    // accL[4], accR[4], P
+  __shared__ double part[2 * kFsCgMax][NP][32];
+  __shared__ unsigned long long hbest[2];
+  const int b0 = half * (32 * kFsHBins) + lane * kFsHBins;
+  int cl[kFsHBins];
+  const int ctot = (int)S[V];
+  {
+    long long cw[kFsHBins];
+    const int64_t oc = (hist_index(p, level, slot) * m + f) * B, os = (hist_index(p, level, sib) * m + f) * B,
+                  op = ((int64_t)par * m + f) * B;
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) {
+      const int b = b0 + i;
+      long long x = 0;
+      if (b < B) {
+        if (derive) { x = pcnt[op + b] - cnt[os + b]; if (store && cg == 0) cnt[oc + b] = (int32_t)x; }
+        else x = cnt[oc + b];
+      }
+      cw[i] = x;
+    }
+    half_scan(cw, half);
+#pragma unroll
+    for (int i = 0; i < kFsHBins; ++i) cl[i] = (int)(half ? (long long)ctot - cw[i] : cw[i]);
+  }
+  const int64_t rowc = (hist_index(p, level, slot) * m + f) * V * B, rows_ = (hist_index(p, level, sib) * m + f) * V * B,
+                rowp = ((int64_t)par * m + f) * V * B;
+  double accL[kFsHBins], accR[kFsHBins];
+#pragma unroll
+  for (int i = 0; i < kFsHBins; ++i) { accL[i] = 0.0; accR[i] = 0.0; }
+  double P = 0.0;
+  auto prefetch = [&](int k) {                           // channel rows two of this warp's iterations ahead
+    if (k >= d) return;
+    const int64_t o = (int64_t)k * B + b0;
+    if (derive) {
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(phist + rowp + o));
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rows_ + o));
+    } else {
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rowc + o));
+    }
+    if (SOFTMAX) {
+      const int64_t oh = (int64_t)(d + k) * B + b0;
+      if (derive) {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(phist + rowp + oh));
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rows_ + oh));
+      } else {
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(hist + rowc + oh));
+      }
+    }
+  };
+  prefetch(cg);
+  prefetch(cg + CG);
+  for (int k = cg; k < d; k += CG) {
+    prefetch(k + 2 * CG);
+    long long gl[kFsHBins];
+    load_row4(gl, b0, hist + rowc + (int64_t)k * B, phist + rowp + (int64_t)k * B, hist + rows_ + (int64_t)k * B,
+              derive, store, B);
+    half_scan(gl, half);
+    const long long G = S[k];
+    if (half) {
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) gl[i] = G - gl[i];
+    }
+    const double sg = (double)scales[k];
+    if (!SOFTMAX) {
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) {
+        const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
+        accL[i] = fma(GL, GL, accL[i]);
+        accR[i] = fma(GR, GR, accR[i]);
+      }
+      const double Gd = (double)G * sg;
+      P = fma(Gd, Gd, P);
+    } else {
+      long long hl[kFsHBins];
+      load_row4(hl, b0, hist + rowc + (int64_t)(d + k) * B, phist + rowp + (int64_t)(d + k) * B,
+                hist + rows_ + (int64_t)(d + k) * B, derive, store, B);
+      half_scan(hl, half);
+      const long long H = S[d + k];
+      if (half) {
+#pragma unroll
+        for (int i = 0; i < kFsHBins; ++i) hl[i] = H - hl[i];
+      }
+      const double sh = (double)scales[d + k];
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) {
+        const double GL = (double)gl[i] * sg, GR = (double)(G - gl[i]) * sg;
+        const double HL = (double)hl[i] * sh, HR = (double)(H - hl[i]) * sh;
+        accL[i] += eq3_pair(GL, HL + lam, GR, HR + lam);
+      }
+      const double Gd = (double)G * sg, Hd = (double)H * sh;
+      P += Gd * Gd / (Hd + lam);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < kFsHBins; ++i) { part[warp][i][lane] = accL[i]; part[warp][kFsHBins + i][lane] = accR[i]; }
+  part[warp][2 * kFsHBins][lane] = P;
+  __syncthreads();
+  if (cg == 0) {
+    for (int g = 1; g < CG; ++g) {                     // fixed order: cg 0, 1, ..., CG-1
+      const int w = 2 * g + half;
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) { accL[i] += part[w][i][lane]; accR[i] += part[w][kFsHBins + i][lane]; }
+      P += part[w][2 * kFsHBins][lane];
+    }
+    uint64_t best = 0;
+    if (half * (32 * kFsHBins) < B) {
+      const int nb = nbins[f];
+      const int64_t fb0 = (int64_t)(p.f_begin + f) * B;
+#pragma unroll
+      for (int i = 0; i < kFsHBins; ++i) {
+        const int b = b0 + i;
+        const long long c = cl[i];
+        if (b < B && b <= nb - 2 && c >= p.min_node && ctot - c >= p.min_node) {
+          double gain;
+          if (!SOFTMAX)
+            gain = 0.5 * (accL[i] / (2.0 * (double)c + lam) + accR[i] / (2.0 * (double)(ctot - c) + lam) -
+                          P / (2.0 * (double)ctot + lam));
+          else
+            gain = 0.5 * (accL[i] - P);
+          if (gain > p.gamma) {
+            const uint64_t key = pack_split_key(gain, fb0 + b);
+            best = key > best ? key : best;
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const uint64_t y = __shfl_xor_sync(0xffffffffu, best, o);
+      best = y > best ? y : best;
+    }
+    if (lane == 0) hbest[half] = best;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint64_t bb = hbest[0] > hbest[1] ? hbest[0] : hbest[1];
+    if (bb) atomicMax((unsigned long long*)&keys[slot], (unsigned long long)bb);
+  }
+}
+
 __global__ void k_zero_u64(uint64_t* p, int64_t n) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) p[i] = 0;
 }
@@ -687,6 +859,21 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
   if (GBDTMO_FS_HALF && !dflt && p->B > 128) {
     // two warps per (node, feature): 2 features x 2 siblings per block, level 0: 4 features
     dim3 grid(level > 0 ? (p->m + 1) / 2 : (p->m + 3) / 4, (unsigned)(level > 0 ? LN / 2 : 1));
+    // few (node, feature) warps for the machine: split the channel loop over CG warp pairs
+    int CG = (int)ctx->fs_channel_groups;               // 0: automatic, 1: off, 2 / 4 / 8: forced
+    if (CG == 0) {
+      const int64_t warps = (int64_t)grid.x * grid.y * kFsWarps, want = (int64_t)ctx->num_sms * 32;
+      CG = warps * 8 <= want ? 8 : warps * 4 <= want ? 4 : warps * 2 <= want ? 2 : 1;
+    }
+    while (CG > 1 && CG > p->d) CG >>= 1;
+    if (GBDTMO_FS_CG_OFF) CG = 1;                        // (A/B builds)
+    if (CG > 1) {
+      auto kc = CG > 4 ? (softmax ? k_find_split_c<true, 8> : k_find_split_c<false, 8>)
+                       : (softmax ? k_find_split_c<true, 4> : k_find_split_c<false, 4>);
+      GB_LAUNCH(kc, dim3((unsigned)LN, (unsigned)p->m), 64 * CG, 0, *p, level, nbins, scales, s, hist, cnt,
+                level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
+      return GBDTMO_OK;
+    }
     auto kern = softmax ? k_find_split_h<true, 3> : channels(*p) <= 16 ? k_find_split_h<false, 4>
                                                                         : k_find_split_h<false, 3>;
     GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt, level > 0 ? parent_hist : hist,

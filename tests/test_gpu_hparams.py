@@ -12,7 +12,7 @@ import pytest
 import torch
 
 from gen import gen
-from tests.gpu_helpers import compare_trees, to_np
+from tests.gpu_helpers import compare_trees, tie_locked_oracle, to_np
 
 pytestmark = pytest.mark.gpu
 
@@ -52,7 +52,7 @@ def _inputs(case, d=None, B=None):
     return w, X, Y
 
 
-def _run(orc, pkg, ctx, w, X, Y, lam, gamma_frac, lr, min_node, hk):
+def _run(orc, pkg, ctx, w, X, Y, lam, gamma_frac, lr, min_node, hk, **kw):
     cuts, nbins, bins = orc.bin_matrix(X, w.B)
     gamma = 0.0
     if gamma_frac:
@@ -63,7 +63,7 @@ def _run(orc, pkg, ctx, w, X, Y, lam, gamma_frac, lr, min_node, hk):
                     min_node=min_node)
     P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=lam, gamma=gamma, lr=lr, min_node=min_node)
     ds = pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B)
-    b = pkg.Booster(ctx, ds, torch.from_numpy(np.ascontiguousarray(Y)).cuda(), P, hist_kernel=hk)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(np.ascontiguousarray(Y)).cuda(), P, hist_kernel=hk, **kw)
     b.fit()
     torch.cuda.synchronize()
     n_leaf_gamma = 0
@@ -109,6 +109,42 @@ GRID = [
 def test_hparam_grid_vs_oracle(orc, pkg, ctx, case, d, B, lam, gfrac, lr, mn, hk):
     w, X, Y = _inputs(case, d, B)
     _run(orc, pkg, ctx, w, X, Y, lam, gfrac, lr, mn, hk)
+
+
+@pytest.mark.parametrize("cg", [1, 2, 4, 8])
+@pytest.mark.parametrize("case,d,lam,gfrac,mn", [("C3s", None, 1.0, 0.0, 20), ("C3s", 3, 0.5, 0.3, 5),
+                                                   ("C2s", None, 1.0, 0.0, 20), ("C2s", 2, 2.5, 0.0, 1),
+                                                   ("C1", None, 0.0, 0.3, 5)])
+def test_channel_split_search_vs_oracle(orc, pkg, ctx, case, d, lam, gfrac, mn, cg):
+    """GBDTMO_OPT_FS_CHANNEL_GROUPS forced to 1 (half-row kernel), 2 and 4 (k_find_split_c: the
+    Eq. (3) sum over outputs split over warp pairs, CG > d clamped): trees, gains, leaves
+    and predictions equal the oracle's at every level, incl. derived children and the last level."""
+    w, X, Y = _inputs(case, d)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    y = Y.astype(np.float64)
+    gamma = 0.0
+    if gfrac:
+        r0 = orc.train(bins, nbins, w.B, y, loss=w.loss, T=1, D=1, lam=lam, gamma=0.0, lr=1.0, min_node=mn)
+        gamma = gfrac * r0["gain"][0][0]
+    ref = orc.train(bins, nbins, w.B, y, loss=w.loss, T=w.T, D=w.D, lam=lam, gamma=gamma, lr=1.0, min_node=mn)
+    P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=lam, gamma=gamma, lr=1.0, min_node=mn)
+    ds = pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B)
+    b = pkg.Booster(ctx, ds, torch.from_numpy(np.ascontiguousarray(Y)).cuda(), P, fs_channel_groups=cg)
+    b.fit()
+    torch.cuda.synchronize()
+    trees = [to_np(t) for t in b.trees]
+    for t in range(w.T):
+        if compare_trees(trees[t], ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]):
+            # a near-tie (min_node 1, binary softmax: symmetric candidates): the tie-locked oracle
+            # (R30) adopts the GPU's choice where the gains tie within 1e-6 and must agree elsewhere
+            pred, ties = tie_locked_oracle(orc, bins, nbins, w.B, y, w.loss, np.zeros_like(y), trees, 0, w.T,
+                                           w.D, lam, gamma, 1.0, mn)
+            assert ties
+            assert np.max(np.abs(b.pred.cpu().numpy() - pred)) <= 1e-4
+            return
+        sp = trees[t]["node_state"] == 1
+        np.testing.assert_allclose(trees[t]["gain"][sp], ref["gain"][t][sp], rtol=1e-6)
+    assert np.max(np.abs(b.pred.cpu().numpy() - ref["pred"])) <= 1e-4
 
 
 def test_gamma_makes_leaves_where_oracle_does(orc, pkg, ctx):

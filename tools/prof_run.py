@@ -17,7 +17,7 @@ from gen import gen  # noqa: E402
 def main():
     wl = sys.argv[1] if len(sys.argv) > 1 else "C5"
     trees = int(sys.argv[2]) if len(sys.argv) > 2 else 2
-    w = gen.WORKLOADS[wl]
+    w = gen.sweep(int(wl[1:])) if wl.startswith("S") else gen.WORKLOADS[wl]
     dev = torch.device("cuda:0")
     ctx = pkg.Context(0)
     X = torch.empty((w.n, w.m), dtype=torch.float32, device=dev)
@@ -32,6 +32,8 @@ def main():
         kw["packed_bins"] = os.environ["PACKED"] == "1"
     if os.environ.get("SMALL_MAX_ROWS") is not None:
         kw["small_max_rows"] = int(os.environ["SMALL_MAX_ROWS"])
+    if os.environ.get("FS_CG") is not None:         # A/B: GBDTMO_OPT_FS_CHANNEL_GROUPS
+        kw["fs_channel_groups"] = int(os.environ["FS_CG"])
     b = pkg.Booster(ctx, ds, Y, P, **kw)
     for _ in range(trees):
         b.step()

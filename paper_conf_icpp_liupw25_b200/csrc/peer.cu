@@ -71,6 +71,10 @@ k_peer_gather(gbdtmo_problem p, int level, PeerView pv, int64_t* __restrict__ xc
   const int64_t total = peer_xchg_count(p), off = peer_xchg_off(p, level) / 8;
   const int64_t pairs = total / 2;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  if (!ok) {          // an expired wait (error word set): no records, every node of the level stays a leaf
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += stride) xchg_out[i] = 0;
+    return;
+  }
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < pairs; i += stride) {
     long long a = 0, b = 0;
     for (int r = 0; r < pv.world; ++r) {

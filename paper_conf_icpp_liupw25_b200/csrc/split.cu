@@ -16,6 +16,9 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_PF
 #define GBDTMO_FS_PF 2           // channels of L2 prefetch ahead in the split search
 #endif
+#ifndef GBDTMO_FS_SOFTMAX_MINB
+#define GBDTMO_FS_SOFTMAX_MINB 4  // resident blocks per SM of the softmax half-row search: 4 (64 registers, 24 B spilled): C2 find_split 1.80 -> 1.70 ms (profiles/r02_ab_fs_softmax_minb4.jsonl)
+#endif
 #ifndef GBDTMO_FS_CG_OFF
 #define GBDTMO_FS_CG_OFF 0       // (A/B) 1: no channel-split search (k_find_split_c)
 #endif
@@ -324,7 +327,7 @@ __device__ __forceinline__ void load_row4(long long (&v)[kFsHBins], int b0, cons
 
 // MINB = resident blocks per SM the kernel is compiled for: 3 (80 registers); MSE problems with at
 // most 16 channels take 4 (64 registers, 8 bytes spilled): C5 9.60 -> 9.27 ms per tree, while C3 / C4
-// lose 3-6% with it (profiles/r02_ab_find_split_minb4.jsonl).  Softmax keeps 3 (2: C2 2.40 -> 2.99 ms).
+// lose 3-6% with it (profiles/r02_ab_find_split_minb4.jsonl).  Softmax takes 4 as well (GBDTMO_FS_SOFTMAX_MINB; 2: C2 2.40 -> 2.99 ms, 4: 1.80 -> 1.70).
 template <bool SOFTMAX, int MINB>
 __global__ void __launch_bounds__(kFsWarps * 32, MINB)
 k_find_split_h(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, const float* __restrict__ scales,
@@ -874,7 +877,7 @@ extern "C" gbdtmo_status gbdtmo_find_split(gbdtmo_ctx c, const gbdtmo_problem* p
                 level > 0 ? parent_hist : hist, level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);
       return GBDTMO_OK;
     }
-    auto kern = softmax ? k_find_split_h<true, 3> : channels(*p) <= 16 ? k_find_split_h<false, 4>
+    auto kern = softmax ? k_find_split_h<true, GBDTMO_FS_SOFTMAX_MINB> : channels(*p) <= 16 ? k_find_split_h<false, 4>
                                                                         : k_find_split_h<false, 3>;
     GB_LAUNCH(kern, grid, kFsWarps * 32, 0, *p, level, nbins, scales, s, hist, cnt, level > 0 ? parent_hist : hist,
               level > 0 ? parent_cnt : cnt, keys, level < p->D - 1 ? 1 : 0);

@@ -5,244 +5,271 @@
 // histograms of B x V entries per feature (C2: 40 KB per feature, 32 MB per node): building,
 // subtracting and re-reading them in HBM costs far more than the rows themselves.  A node marked
 // SMALL by the plan (both children of its parent fit GBDTMO_OPT_SMALL_MAX_ROWS) is searched
-// directly from its rows instead, and never materialised:
-//   - one CTA per (node, block of features) stages the node's row ids and q rows in shared memory;
-//   - one warp per feature counting-sorts the node's rows by bin (shared counters, in-place
-//     exclusive scan), then walks them in bin order with lanes = outputs, accumulating the exact
-//     int64 G_L (and H_L) prefix sums from the staged q rows;
-//   - at every bin boundary, i.e. only for bins present in the node (an empty bin gives the same
-//     partition as its predecessor), each output lane writes its Eq. (3) term to a
-//     kCand-candidate buffer; a full buffer is reduced with lanes = candidates (no shuffles on the
-//     walk), and the best packed key per CTA is max-reduced into keys[slot] — the same key and
-//     tie rule as k_find_split, so the chosen split is the same.
+// directly from its rows instead, and never materialised (k_seg_search below).
 #include "common.cuh"
 
 namespace gbdtmo {
 
-// A warp searches G features at once (G = 32 / d rounded down to 1, 2, 3, 4 or 8): lanes are
-// (feature group g, output k), so a d = 10 softmax node keeps 30 of 32 lanes busy instead of 10.
-constexpr int kSortWarpsMax = 16;
+// Segmented-scan search (round 2).  It replaces a serial walk (one lane per output stepping through
+// the node's rows in bin order: ~470 dependent steps at C2's deepest level, 3 features' buffers per
+// warp, one 8-warp CTA per SM: 12.5% occupancy, 38% issue, `profiles/r02_ncu_small_C2.txt`; 3x
+// slower per level, `profiles/r02c_ncu_small_seg_C2.txt`).  A warp takes ONE feature at a time and
+// its lanes take positions of the node's rows in bin order:
+//   - counting sort by bin (shared counters), the sorted row indices stored lane-major
+//     (sidxT[i][lane] = row at position lane * PL + i, PL = ceil(R / 32): conflict-free reads);
+//   - candidates = positions j < R - 1 ending a bin (sb[j] != sb[j + 1], R27) that are valid
+//     (bin <= nb - 2, both sides >= min_node), compacted per warp (cpos, cbin);
+//   - per output k: each lane sums q[., k] (and q[., d + k]) over its PL positions, writing the
+//     running sum at its candidates; a warp scan of the lane totals turns those into the exact
+//     int64 prefix sums G_L (H_L); then lanes take candidates round-robin and add the output's
+//     Eq. (3) term in the same fp64 order as k_find_split_h (acc = fma(GL, GL, acc) / eq3_pair),
+//     with the parent term P summed the same way, so gains and keys are bit-identical to the
+//     histogram path's.
+// The CTA stages the node's row ids and q rows once for all the features its warps walk.
+constexpr int kSegWarps = 16;
+constexpr int kSegCand = 256;          // candidates per (node, feature) <= distinct bins - 1 <= 255
 
-__host__ __device__ inline int small_groups(int d) { return d <= 4 ? 8 : d <= 8 ? 4 : d <= 10 ? 3 : d <= 16 ? 2 : 1; }
-__host__ __device__ inline int small_warps(int G) { return G > 1 ? 8 : 16; }
-__host__ __device__ inline int small_cpg(int G) { return G > 1 ? 32 / G : 16; }   // buffered candidates per group
-
-struct SmallLayout {
-  int G, W, CPG;                   // features per warp, warps per CTA, candidates per group
-  int dp;                          // doubles per buffered candidate (d rounded up to odd: conflict-free reads)
-  int o_qs, o_warps;               // CTA-shared: row ids [rc] i32 at 0, q rows [rc][V] i32 at o_qs
-  int g_bytes;                     // per (warp, group): counts[256] u32 | sidx [rc] u16 | bk [rc] u8 | sb [rc + 8] u8
-  int o_sidx, o_bk, o_sb;          // offsets inside a group's region
-  int o_cand, o_cbin, warp_bytes;  // per warp: G regions, then cand [G][CPG][dp] f64, cbin [G][CPG] i32
-  int bytes;                       // dynamic shared memory of one CTA
+struct SegLayout {
+  int rc, V;
+  int o_qs, o_warps, warp_bytes, bytes;
+  // per warp: cnt[256] u32 | candG[256] i64 | aux[256] (softmax candH i64 / MSE accR f64) |
+  //           acc[256] f64 | cpos[256] u16 | cbin[256] u8 | bk[rc] u8 | sb[rc + 8] u8 | sidxT[rc32] u16
+  int o_cnt, o_candG, o_aux, o_acc, o_cpos, o_cbin, o_bk, o_sb, o_sidx;
 };
 
-__host__ __device__ inline SmallLayout small_layout(const gbdtmo_problem& p, int64_t rcap) {
-  SmallLayout L;
-  const int rc = (int)((rcap + 7) / 8 * 8);
-  L.G = small_groups(p.d);
-  L.W = small_warps(L.G);
-  L.CPG = small_cpg(L.G);
-  L.dp = p.d | 1;
-  L.o_qs = 4 * rc;
-  L.o_warps = L.o_qs + 4 * channels(p) * rc;
-  L.o_sidx = 1024;
-  L.o_bk = L.o_sidx + 2 * rc;
-  L.o_sb = L.o_bk + rc;
-  L.g_bytes = (L.o_sb + rc + 8 + 7) / 8 * 8;
-  L.o_cand = L.G * L.g_bytes;
-  L.o_cbin = L.o_cand + 8 * L.G * L.CPG * L.dp;
-  L.warp_bytes = L.o_cbin + 4 * L.G * L.CPG;
-  L.bytes = L.o_warps + L.W * L.warp_bytes;
+__host__ __device__ inline SegLayout seg_layout(const gbdtmo_problem& p, int64_t rcap) {
+  SegLayout L;
+  L.rc = (int)((rcap + 31) / 32 * 32);
+  L.V = channels(p);
+  L.o_qs = 4 * L.rc;
+  L.o_warps = (L.o_qs + 4 * L.V * L.rc + 15) / 16 * 16;
+  L.o_cnt = 0;
+  L.o_candG = L.o_cnt + 4 * 256;
+  L.o_aux = L.o_candG + 8 * kSegCand;
+  L.o_acc = L.o_aux + 8 * kSegCand;
+  L.o_cpos = L.o_acc + 8 * kSegCand;
+  L.o_cbin = L.o_cpos + 2 * kSegCand;
+  L.o_bk = L.o_cbin + kSegCand;
+  L.o_sb = L.o_bk + L.rc;
+  L.o_sidx = L.o_sb + L.rc + 16;
+  L.warp_bytes = (L.o_sidx + 2 * L.rc + 15) / 16 * 16;
+  L.bytes = L.o_warps + kSegWarps * L.warp_bytes;
   return L;
 }
 
-__host__ __device__ inline int64_t small_cap(const gbdtmo_problem& p) {
-  const SmallLayout L0 = small_layout(p, 0);
-  int64_t r = (kHistSmemBudget - L0.bytes) / (4 + 4 * channels(p) + L0.W * L0.G * 4) - 8;
-  if (r > 65535) r = 65535;                                    // 16-bit local row indices
+__host__ __device__ inline int64_t seg_cap(const gbdtmo_problem& p) {
+  const int V = channels(p);
+  // bytes(rc) = 4 rc (1 + V) + W (7936 + 4 rc + 16) (+ alignment)
+  const int64_t fixed = (int64_t)kSegWarps * (4 * 256 + 3 * 8 * kSegCand + 2 * kSegCand + kSegCand + 16) + 64;
+  int64_t r = (kHistSmemBudget - fixed) / (4 * (1 + V) + 4 * kSegWarps);
+  r = r / 32 * 32;
+  if (r > 1024) r = 1024;                          // <= 32 positions per lane (one candidate bit each)
   return r < 0 ? 0 : r;
 }
 
-__device__ __forceinline__ double warp_sum_d(double x) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-  return x;
-}
-
-template <bool SOFTMAX, int G>
-__global__ void __launch_bounds__(G > 1 ? 256 : 512)
-k_sort_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ bins,
-              const int32_t* __restrict__ q, const int32_t* __restrict__ rows, int use_rows,
-              const int32_t* __restrict__ nbins, const float* __restrict__ scales, State s,
-              uint64_t* __restrict__ keys) {
+template <bool SOFTMAX>
+__global__ void __launch_bounds__(kSegWarps * 32)
+k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ bins,
+             const int32_t* __restrict__ q, const int32_t* __restrict__ rows, int use_rows,
+             const int32_t* __restrict__ nbins, const float* __restrict__ scales, State s,
+             uint64_t* __restrict__ keys) {
   extern __shared__ __align__(16) unsigned char smraw[];
-  __shared__ unsigned long long sh_best[kSortWarpsMax];
+  __shared__ unsigned long long sh_best[kSegWarps];
   if ((int)blockIdx.y >= s.misc[MISC_SNODE_COUNT]) return;
   const int4 nd = s.snodes[blockIdx.y];
   const int64_t h = (int64_t(1) << level) - 1 + nd.x;
-  const int r = nd.z - nd.y;
+  const int R = nd.z - nd.y;
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const SmallLayout L = small_layout(p, rcap);
-  constexpr int CPG = G > 1 ? 32 / G : 16;
-  const int W = L.W;
+  const SegLayout L = seg_layout(p, rcap);
   int32_t* rid = reinterpret_cast<int32_t*>(smraw);
   int32_t* qs = reinterpret_cast<int32_t*>(smraw + L.o_qs);
   unsigned char* wb = smraw + L.o_warps + warp * L.warp_bytes;
-  double* cand = reinterpret_cast<double*>(wb + L.o_cand);          // [G][CPG][dp]
-  int32_t* cbin = reinterpret_cast<int32_t*>(wb + L.o_cbin);        // [G][CPG]
-  // stage the node's row ids and q rows (shared by every feature of this CTA)
-  for (int i = threadIdx.x; i < r; i += blockDim.x) rid[i] = use_rows ? rows[nd.y + i] : nd.y + i;
+  uint32_t* cnt = reinterpret_cast<uint32_t*>(wb + L.o_cnt);
+  long long* candG = reinterpret_cast<long long*>(wb + L.o_candG);
+  long long* candH = reinterpret_cast<long long*>(wb + L.o_aux);      // softmax
+  double* accR = reinterpret_cast<double*>(wb + L.o_aux);             // MSE
+  double* acc = reinterpret_cast<double*>(wb + L.o_acc);
+  uint16_t* cpos = reinterpret_cast<uint16_t*>(wb + L.o_cpos);
+  unsigned char* cbin = wb + L.o_cbin;
+  unsigned char* bk = wb + L.o_bk;
+  unsigned char* sb = wb + L.o_sb;
+  uint16_t* sidxT = reinterpret_cast<uint16_t*>(wb + L.o_sidx);
+  for (int i = threadIdx.x; i < R; i += blockDim.x) rid[i] = use_rows ? rows[nd.y + i] : nd.y + i;
   __syncthreads();
-  for (int e = threadIdx.x; e < r * V; e += blockDim.x) {
+  for (int e = threadIdx.x; e < R * V; e += blockDim.x) {
     const int i = e / V, c = e - i * V;
     qs[e] = __ldg(&q[(int64_t)rid[i] * V + c]);
   }
   __syncthreads();
-  // lanes: (group g, output k)
-  const int g = G > 1 ? lane / d : 0, k = G > 1 ? lane - g * d : lane;
-  const bool lon = g < G && k < d;
-  // node totals (exact) and the parent term of Eq. (3): the same for every feature
   const int64_t* S = s.node_sum + h * (V + 1);
   const long long C = S[V];
   const double lam = p.lambda;
-  const bool k0 = lane < d;                               // lanes 0..d-1 compute the parent term once
-  const double sg = lon ? (double)scales[k] : 0.0;
-  const double sh = (SOFTMAX && lon) ? (double)scales[d + k] : 0.0;
-  const long long Gt = lon ? S[k] : 0, Ht = (SOFTMAX && lon) ? S[d + k] : 0;
-  double P;
-  {
-    const double sg0 = k0 ? (double)scales[lane] : 0.0, sh0 = (SOFTMAX && k0) ? (double)scales[d + lane] : 0.0;
-    const double Gd0 = k0 ? (double)S[lane] * sg0 : 0.0;
-    const double Hd0 = (SOFTMAX && k0) ? (double)S[d + lane] * sh0 : 0.0;
-    P = SOFTMAX ? warp_sum_d(k0 ? Gd0 * Gd0 / (Hd0 + lam) : 0.0) : warp_sum_d(Gd0 * Gd0) / (2.0 * (double)C + lam);
+  // parent term, summed over outputs in k_find_split_h's order
+  double P = 0.0;
+  for (int k = 0; k < d; ++k) {
+    const double Gd = (double)S[k] * (double)scales[k];
+    if (SOFTMAX) {
+      const double Hd = (double)S[d + k] * (double)scales[d + k];
+      P += Gd * Gd / (Hd + lam);
+    } else {
+      P = fma(Gd, Gd, P);
+    }
   }
-  const int32_t* qg = qs + (lon ? k : 0);
-  const int32_t* qh = qs + (lon ? d + k : 0);
+  const int PL = (R + 31) >> 5;                    // positions per lane
   uint64_t best = 0;
-  for (int f0 = (blockIdx.x * W + warp) * G; f0 < m; f0 += gridDim.x * W * G) {
-    // ---- counting sort of the node's rows by bin, one feature per group
-#pragma unroll 1
-    for (int gg = 0; gg < G; ++gg) {
-      const int f = f0 + gg;
-      if (f >= m) break;
-      unsigned char* gr = wb + gg * L.g_bytes;
-      uint32_t* cnt = reinterpret_cast<uint32_t*>(gr);
-      uint16_t* sidx = reinterpret_cast<uint16_t*>(gr + L.o_sidx);
-      unsigned char* bk = gr + L.o_bk;
-      unsigned char* sb = gr + L.o_sb;
+  for (int f = blockIdx.x * kSegWarps + warp; f < m; f += gridDim.x * kSegWarps) {
+    // ---- counting sort of the node's rows by bin
 #pragma unroll
-      for (int t = 0; t < 8; ++t) cnt[lane * 8 + t] = 0;
+    for (int t = 0; t < 8; ++t) cnt[lane * 8 + t] = 0;
+    __syncwarp();
+    for (int i0 = 0; i0 < R; i0 += 128) {
+      int bv[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int i = i0 + u * 32 + lane;
+        bv[u] = i < R ? (int)__ldg(&bins[(int64_t)rid[i] * p.ld_bins + f]) : -1;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (bv[u] >= 0) { bk[i0 + u * 32 + lane] = (unsigned char)bv[u]; atomicAdd(&cnt[bv[u]], 1u); }
+    }
+    __syncwarp();
+    {
+      uint32_t v[8], run = 0;
+#pragma unroll
+      for (int t = 0; t < 8; ++t) { v[t] = run; run += cnt[lane * 8 + t]; }
+      uint32_t x = run;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      const uint32_t ex = x - run;
       __syncwarp();
-      for (int i0 = 0; i0 < r; i0 += 128) {
-        int bv[4];
+#pragma unroll
+      for (int t = 0; t < 8; ++t) cnt[lane * 8 + t] = ex + v[t];
+    }
+    __syncwarp();
+    for (int i = lane; i < R; i += 32) {
+      const int b = bk[i];
+      const uint32_t pos = atomicAdd(&cnt[b], 1u);
+      sb[pos] = (unsigned char)b;
+      const uint32_t ow = pos / PL, oi = pos - ow * PL;
+      sidxT[oi * 32 + ow] = (uint16_t)i;
+    }
+    __syncwarp();
+    // ---- candidates of this lane's positions [lane PL, lane PL + PL), compacted per warp
+    const int nb = nbins[f];
+    const int p0 = lane * PL;
+    uint32_t cm = 0;                               // bit i: position p0 + i is a candidate
+    for (int i = 0; i < PL; ++i) {
+      const int j = p0 + i;
+      if (j < R - 1) {
+        const int b = sb[j];
+        const long long CL = j + 1;
+        if (b != (int)sb[j + 1] && b <= nb - 2 && CL >= p.min_node && C - CL >= p.min_node) cm |= 1u << i;
+      }
+    }
+    int cb = __popc(cm), ctot;
+    {
+      int x = cb;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      ctot = __shfl_sync(0xffffffffu, x, 31);
+      cb = x - cb;                                 // this lane's first candidate index
+    }
+    if (ctot == 0) continue;                       // (warp-uniform)
+    {
+      int ci = cb;
+      for (uint32_t mm = cm; mm; mm &= mm - 1) {
+        const int i = __ffs(mm) - 1;
+        cpos[ci] = (uint16_t)(p0 + i);
+        cbin[ci] = sb[p0 + i];
+        ++ci;
+      }
+    }
+    for (int c = lane; c < ctot; c += 32) { acc[c] = 0.0; if (!SOFTMAX) accR[c] = 0.0; }
+    __syncwarp();
+    // ---- per output: exact prefix sums at the candidates, then the Eq. (3) terms
+    for (int k = 0; k < d; ++k) {
+      long long g = 0, hh = 0;
+      int ci = cb;
+      const int pe = min(PL, R - p0);              // this lane's positions
+      for (int i0 = 0; i0 < pe; i0 += 4) {         // 4 independent row loads in flight
+        int qg[4], qh[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          const int i = i0 + u * 32 + lane;
-          bv[u] = i < r ? (int)bins[(int64_t)rid[i] * p.ld_bins + f] : -1;
+          const int r = i0 + u < pe ? (int)sidxT[(i0 + u) * 32 + lane] : -1;
+          qg[u] = r >= 0 ? qs[r * V + k] : 0;
+          qh[u] = (SOFTMAX && r >= 0) ? qs[r * V + d + k] : 0;
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-          if (bv[u] >= 0) {
-            bk[i0 + u * 32 + lane] = (unsigned char)bv[u];
-            atomicAdd(&cnt[bv[u]], 1u);
+          g += qg[u];
+          if (SOFTMAX) hh += qh[u];
+          if ((cm >> (i0 + u)) & 1u) {
+            candG[ci] = g;
+            if (SOFTMAX) candH[ci] = hh;
+            ++ci;
           }
         }
       }
-      __syncwarp();
-      {
-        uint32_t v[8], run = 0;
+      // exclusive offsets of the lane totals
+      long long og = g, oh = hh;
 #pragma unroll
-        for (int t = 0; t < 8; ++t) { v[t] = run; run += cnt[lane * 8 + t]; }
-        uint32_t x = run;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-          if (lane >= o) x += y;
-        }
-        const uint32_t ex = x - run;
-        __syncwarp();
-#pragma unroll
-        for (int t = 0; t < 8; ++t) cnt[lane * 8 + t] = ex + v[t];
+      for (int o = 1; o < 32; o <<= 1) {
+        const long long yg = __shfl_up_sync(0xffffffffu, og, o);
+        const long long yh = SOFTMAX ? __shfl_up_sync(0xffffffffu, oh, o) : 0;
+        if (lane >= o) { og += yg; if (SOFTMAX) oh += yh; }
       }
+      og -= g;
+      oh -= hh;
+      for (int c = cb; c < ci; ++c) { candG[c] += og; if (SOFTMAX) candH[c] += oh; }
       __syncwarp();
-      for (int i = lane; i < r; i += 32) {
-        const int b = bk[i];
-        const uint32_t pos = atomicAdd(&cnt[b], 1u);
-        sidx[pos] = (uint16_t)i;
-        sb[pos] = (unsigned char)b;
+      const long long G = S[k];
+      const double sg = (double)scales[k];
+      if (SOFTMAX) {
+        const long long H = S[d + k];
+        const double sh = (double)scales[d + k];
+        for (int c = lane; c < ctot; c += 32) {
+          const long long gl = candG[c], hl = candH[c];
+          const double GL = (double)gl * sg, GR = (double)(G - gl) * sg;
+          const double HL = (double)hl * sh, HR = (double)(H - hl) * sh;
+          acc[c] += eq3_pair(GL, HL + lam, GR, HR + lam);
+        }
+      } else {
+        for (int c = lane; c < ctot; c += 32) {
+          const long long gl = candG[c];
+          const double GL = (double)gl * sg, GR = (double)(G - gl) * sg;
+          acc[c] = fma(GL, GL, acc[c]);
+          accR[c] = fma(GR, GR, accR[c]);
+        }
       }
       __syncwarp();
     }
-    // ---- walk in bin order, all groups together: after row j of group g's order, "bin <= sb[j]"
-    //      is a candidate when sb[j + 1] differs (only bins present in the node, R27)
-    const int fg = f0 + g;
-    const bool gon = lon && fg < m;
-    const unsigned char* gr = wb + (gon ? g : 0) * L.g_bytes;
-    const uint16_t* sidx = reinterpret_cast<const uint16_t*>(gr + L.o_sidx);
-    const unsigned char* sb = gr + L.o_sb;
-    const int nb = gon ? nbins[fg] : 0;
-    long long GL = 0, HL = 0;
-    int nc = 0;                                           // candidates buffered for this lane's group
-    auto flush = [&]() {
-      __syncwarp();
-      // lanes = (group, candidate): lane L2 = gg * CPG + c
-      const int gg = lane / CPG, c = lane - gg * CPG;
-      const int ncg = __shfl_sync(0xffffffffu, nc, gg < G ? gg * d : 0);
-      if (gg < G && c < ncg) {
-        double t = 0.0;
-        const double* cd = cand + ((int64_t)gg * CPG + c) * L.dp;
-        for (int kk = 0; kk < d; ++kk) t += cd[kk];
-        const double gain = 0.5 * (t - P);
-        if (gain > p.gamma) {
-          const int64_t fbg = (int64_t)(p.f_begin + f0 + gg) * B;
-          const uint64_t key = pack_split_key(gain, fbg + cbin[gg * CPG + c]);
-          best = key > best ? key : best;
-        }
-      }
-      __syncwarp();
-      nc = 0;
-    };
-    for (int j0 = 0; j0 < r - 1; j0 += 4) {
-      int ix[4];
-      int gv[4], hv[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) ix[u] = (gon && j0 + u < r - 1) ? (int)sidx[j0 + u] : -1;
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        gv[u] = ix[u] >= 0 ? qg[ix[u] * V] : 0;
-        hv[u] = (SOFTMAX && ix[u] >= 0) ? qh[ix[u] * V] : 0;
-      }
-      const uint32_t b4 = *reinterpret_cast<const uint32_t*>(sb + j0);     // sb is 8-aligned, j0 % 4 == 0
-      const uint32_t n4 = (uint32_t)sb[j0 + 4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        GL += gv[u];
-        if (SOFTMAX) HL += hv[u];
-        const int b = (b4 >> (8 * u)) & 0xff;
-        const int bn = u < 3 ? (int)((b4 >> (8 * (u + 1))) & 0xff) : (int)n4;
-        const long long CL = j0 + u + 1;
-        if (ix[u] >= 0 && b != bn && b <= nb - 2 && CL >= p.min_node && C - CL >= p.min_node) {
-          const double gl = (double)GL * sg, gr_ = (double)(Gt - GL) * sg;
-          double t;
-          if (SOFTMAX) {
-            t = eq3_pair(gl, (double)HL * sh + lam, gr_, (double)(Ht - HL) * sh + lam);
-          } else {
-            t = gl * gl / (2.0 * (double)CL + lam) + gr_ * gr_ / (2.0 * (double)(C - CL) + lam);
-          }
-          cand[((int64_t)g * CPG + nc) * L.dp + k] = t;
-          if (k == 0) cbin[g * CPG + nc] = b;
-          ++nc;
-        }
-        // a group whose buffer is full makes the whole warp reduce (lanes = (group, candidate))
-        if (__any_sync(0xffffffffu, nc == CPG)) flush();
+    // ---- gains and keys (k_find_split_h's formulas)
+    const int64_t fbg = (int64_t)(p.f_begin + f) * B;
+    for (int c = lane; c < ctot; c += 32) {
+      const long long CL = (long long)cpos[c] + 1;
+      double gain;
+      if (SOFTMAX)
+        gain = 0.5 * (acc[c] - P);
+      else
+        gain = 0.5 * (acc[c] / (2.0 * (double)CL + lam) + accR[c] / (2.0 * (double)(C - CL) + lam) -
+                      P / (2.0 * (double)C + lam));
+      if (gain > p.gamma) {
+        const uint64_t key = pack_split_key(gain, fbg + cbin[c]);
+        best = key > best ? key : best;
       }
     }
-    if (__any_sync(0xffffffffu, nc > 0)) flush();
+    __syncwarp();
   }
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {                     // lanes hold their candidates' bests
+  for (int o = 16; o > 0; o >>= 1) {
     const unsigned long long y = __shfl_xor_sync(0xffffffffu, (unsigned long long)best, o);
     best = y > best ? y : best;
   }
@@ -250,13 +277,13 @@ k_sort_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__
   __syncthreads();
   if (threadIdx.x == 0) {
     uint64_t bb = 0;
-    for (int w = 0; w < W; ++w) bb = sh_best[w] > bb ? sh_best[w] : bb;
+    for (int w = 0; w < kSegWarps; ++w) bb = sh_best[w] > bb ? sh_best[w] : bb;
     if (bb) atomicMax((unsigned long long*)&keys[nd.x], (unsigned long long)bb);
   }
 }
 
-bool small_supported(const gbdtmo_problem& p) { return p.d <= 32 && small_cap(p) >= 64; }
-int64_t small_rows_cap(const gbdtmo_problem& p) { return small_cap(p); }
+bool small_supported(const gbdtmo_problem& p) { return p.B <= 256 && seg_cap(p) >= 64; }
+int64_t small_rows_cap(const gbdtmo_problem& p) { return seg_cap(p); }
 
 }  // namespace gbdtmo
 
@@ -274,29 +301,23 @@ extern "C" gbdtmo_status gbdtmo_search_small(gbdtmo_ctx c, const gbdtmo_problem*
   GB_CHECK_ARG(bins && q && nbins && scales && state && keys, "null pointer");
   const int64_t rcap = small_rows(ctx, *p);
   if (rcap <= 0) return GBDTMO_OK;                          // no node is ever marked SMALL
-  const SmallLayout L = small_layout(*p, rcap);
   State s = state_view(*p, state);
   const int32_t* rows = (level & 1) ? s.rows1 : s.rows0;
   const int use_rows = level > 0;
   const int64_t LN = int64_t(1) << level;
-  // feature blocks per node: enough CTAs for ~3 waves of resident CTAs, at most one warp per G features
-  const int fb_max = (p->m + L.W * L.G - 1) / (L.W * L.G);
-  const int per_sm = L.bytes > 0 ? (int)((ctx->max_smem_optin - 1024) / (L.bytes + 1024)) : 1;
-  int64_t fb = (3LL * ctx->num_sms * (per_sm < 1 ? 1 : per_sm) + LN - 1) / LN;
+  const bool sm = p->loss == GBDTMO_LOSS_SOFTMAX;
+  const SegLayout L = seg_layout(*p, rcap);
+  // feature blocks per node: ~8 waves of resident CTAs over the level's (at most LN) small nodes,
+  // so nodes of different sizes balance (ncu at 2.6 waves: 46% issue, idle SMs in the tail)
+  const int per_sm = (int)((ctx->max_smem_optin) / (L.bytes + 1024));
+  int64_t fb = (8LL * ctx->num_sms * (per_sm < 1 ? 1 : per_sm) + LN - 1) / LN;
+  const int64_t fb_max = (p->m + kSegWarps - 1) / kSegWarps;
   if (fb > fb_max) fb = fb_max;
   if (fb < 1) fb = 1;
-  const bool sm = p->loss == GBDTMO_LOSS_SOFTMAX;
-  decltype(&k_sort_search<true, 1>) kern;
-  switch (L.G) {
-    case 8: kern = sm ? k_sort_search<true, 8> : k_sort_search<false, 8>; break;
-    case 4: kern = sm ? k_sort_search<true, 4> : k_sort_search<false, 4>; break;
-    case 3: kern = sm ? k_sort_search<true, 3> : k_sort_search<false, 3>; break;
-    case 2: kern = sm ? k_sort_search<true, 2> : k_sort_search<false, 2>; break;
-    default: kern = sm ? k_sort_search<true, 1> : k_sort_search<false, 1>; break;
-  }
-  static unsigned long long attr_mask[2][9] = {};
-  smem_optin_once(ctx, kern, attr_mask[sm][L.G], ctx->max_smem_optin - 1024);
-  GB_LAUNCH(kern, dim3((unsigned)fb, (unsigned)LN), L.W * 32, L.bytes, *p, level, (int)rcap, bins, q, rows,
+  auto kern = sm ? k_seg_search<true> : k_seg_search<false>;
+  static unsigned long long seg_mask[2] = {};
+  smem_optin_once(ctx, kern, seg_mask[sm], ctx->max_smem_optin - 1024);
+  GB_LAUNCH(kern, dim3((unsigned)fb, (unsigned)LN), kSegWarps * 32, L.bytes, *p, level, (int)rcap, bins, q, rows,
             use_rows, nbins, scales, s, keys);
   return GBDTMO_OK;
 }

@@ -26,6 +26,10 @@ namespace gbdtmo {
 //     with the parent term P summed the same way, so gains and keys are bit-identical to the
 //     histogram path's.
 // The CTA stages the node's row ids and q rows once for all the features its warps walk.
+#ifndef GBDTMO_BOUNDS_CHECK
+#define GBDTMO_BOUNDS_CHECK 0  // (debug builds) trap on any out-of-range shared-memory index below
+#endif
+#define SEG_CHECK(cond) do { if (GBDTMO_BOUNDS_CHECK && !(cond)) __trap(); } while (0)
 constexpr int kSegWarps = 16;
 constexpr int kSegCand = 256;          // candidates per (node, feature) <= distinct bins - 1 <= 255
 
@@ -82,6 +86,7 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
   const int V = channels(p), B = p.B, m = p.m, d = p.d;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const SegLayout L = seg_layout(p, rcap);
+  SEG_CHECK(R >= 0 && R <= rcap && (R + 31) / 32 <= 32);
   int32_t* rid = reinterpret_cast<int32_t*>(smraw);
   int32_t* qs = reinterpret_cast<int32_t*>(smraw + L.o_qs);
   unsigned char* wb = smraw + L.o_warps + warp * L.warp_bytes;
@@ -132,7 +137,11 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u)
-        if (bv[u] >= 0) { bk[i0 + u * 32 + lane] = (unsigned char)bv[u]; atomicAdd(&cnt[bv[u]], 1u); }
+        if (bv[u] >= 0) {
+          SEG_CHECK(i0 + u * 32 + lane < L.rc && bv[u] < 256);
+          bk[i0 + u * 32 + lane] = (unsigned char)bv[u];
+          atomicAdd(&cnt[bv[u]], 1u);
+        }
     }
     __syncwarp();
     {
@@ -156,6 +165,7 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
       const uint32_t pos = atomicAdd(&cnt[b], 1u);
       sb[pos] = (unsigned char)b;
       const uint32_t ow = pos / PL, oi = pos - ow * PL;
+      SEG_CHECK(pos < (uint32_t)R && ow < 32 && oi * 32 + ow < (uint32_t)L.rc);
       sidxT[oi * 32 + ow] = (uint16_t)i;
     }
     __syncwarp();
@@ -187,6 +197,7 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
       int ci = cb;
       for (uint32_t mm = cm; mm; mm &= mm - 1) {
         const int i = __ffs(mm) - 1;
+        SEG_CHECK(ci < kSegCand && p0 + i < R - 1);
         cpos[ci] = (uint16_t)(p0 + i);
         cbin[ci] = sb[p0 + i];
         ++ci;
@@ -204,6 +215,7 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
           const int r = i0 + u < pe ? (int)sidxT[(i0 + u) * 32 + lane] : -1;
+          SEG_CHECK(r < R);
           qg[u] = r >= 0 ? qs[r * V + k] : 0;
           qh[u] = (SOFTMAX && r >= 0) ? qs[r * V + d + k] : 0;
         }

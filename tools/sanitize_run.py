@@ -4,7 +4,8 @@
 case: C1 | C3s | C2s;  variant: k0 (row-pair smem), k1 (diagonal), k2 (TMA-staged), gmem (global
 atomics for every node), small (sort-and-segment small nodes), sparse (default-bin skip), graph
 (CUDA-graph replay), predict (gbdtmo_predict), binhost (train() from a pinned host matrix:
-gbdtmo_bin_host strip uploads on the context's copy stream), packed (tile-packed bins).  Prints
+gbdtmo_bin_host strip uploads on the context's copy stream), packed (tile-packed bins), cg2 / cg8
+(channel-split split search forced to 2 / 8 warp pairs).  Prints
 the max |pred - oracle| (parity still holds under the tool)."""
 import os
 import sys
@@ -36,7 +37,8 @@ def main():
               gmem=dict(gmem_max_rows=1 << 30, small_max_rows=0),
               small=dict(small_max_rows=4000, gmem_max_rows=0),
               sparse=dict(sparse_default=True, hist_kernel=0),
-              graph=dict(), predict=dict(), binhost=dict(), packed=dict(packed_bins=True, hist_kernel=0))[var]
+              graph=dict(), predict=dict(), binhost=dict(), packed=dict(packed_bins=True, hist_kernel=0),
+              cg8=dict(fs_channel_groups=8), cg2=dict(fs_channel_groups=2))[var]
     P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
     if var == "binhost":
         b = pkg.train(torch.from_numpy(X).pin_memory(), torch.from_numpy(Y), P, ctx=ctx)

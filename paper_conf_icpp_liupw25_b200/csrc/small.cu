@@ -102,9 +102,26 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
   uint16_t* sidxT = reinterpret_cast<uint16_t*>(wb + L.o_sidx);
   for (int i = threadIdx.x; i < R; i += blockDim.x) rid[i] = use_rows ? rows[nd.y + i] : nd.y + i;
   __syncthreads();
-  for (int e = threadIdx.x; e < R * V; e += blockDim.x) {
-    const int i = e / V, c = e - i * V;
-    qs[e] = __ldg(&q[(int64_t)rid[i] * V + c]);
+  // q rows of the node: 8 independent loads in flight per thread (the CTA waits on this once)
+  for (int e0 = threadIdx.x; e0 < R * V; e0 += 8 * blockDim.x) {
+    int v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = e0 + u * blockDim.x;
+      if (e < R * V) {
+        const int i = e / V, c = e - i * V;
+        v[u] = __ldg(&q[(int64_t)rid[i] * V + c]);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int e = e0 + u * blockDim.x;
+      if (e < R * V) {
+        // softmax: (g_k, h_k) interleaved, one 8-byte load per (row, output) in the walk
+        const int i = e / V, c = e - i * V;
+        qs[SOFTMAX ? i * V + 2 * (c < d ? c : c - d) + (c < d ? 0 : 1) : e] = v[u];
+      }
+    }
   }
   __syncthreads();
   const int64_t* S = s.node_sum + h * (V + 1);
@@ -216,8 +233,14 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
         for (int u = 0; u < 4; ++u) {
           const int r = i0 + u < pe ? (int)sidxT[(i0 + u) * 32 + lane] : -1;
           SEG_CHECK(r < R);
-          qg[u] = r >= 0 ? qs[r * V + k] : 0;
-          qh[u] = (SOFTMAX && r >= 0) ? qs[r * V + d + k] : 0;
+          if (SOFTMAX) {
+            const int2 gh = r >= 0 ? *reinterpret_cast<const int2*>(qs + r * V + 2 * k) : make_int2(0, 0);
+            qg[u] = gh.x;
+            qh[u] = gh.y;
+          } else {
+            qg[u] = r >= 0 ? qs[r * V + k] : 0;
+            qh[u] = 0;
+          }
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {

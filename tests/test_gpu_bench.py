@@ -36,3 +36,31 @@ def test_bench_reference_arm():
     j = _run(["--impl", "reference", "--workload", "C1", "--steps", "1", "--warmup", "1"])
     assert j["impl"] == "reference" and j["value"] > 0
     assert j["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_bench_two_ranks_gloo():
+    """The N > 1 launch the driver uses (torch.distributed.run, one JSON line from rank 0, max over
+    ranks), with gloo and the collective exchange so the two ranks can share this one GPU: a smoke
+    test of bench.py's multi-rank plumbing, not a measurement."""
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29571", os.path.join(ROOT, "bench.py"),
+                        "--gpus", "2", "--steps", "2", "--warmup", "3", "--workload", "C1", "--backend", "gloo",
+                        "--exchange", "collective", "--no-cpu-baseline"],
+                       capture_output=True, text=True, cwd=ROOT, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    j = json.loads(lines[0])
+    assert j["n_gpus"] == 2 and j["value"] > 0 and j["e2e"]["value"] > 0
+    assert "feature-partition x2" in j["config"]["parallelism"]
+
+
+def test_bench_reference_two_ranks():
+    """--impl reference under torch.distributed.run: rank 0 alone prints the line, the others exit 0."""
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29573", os.path.join(ROOT, "bench.py"),
+                        "--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "1", "--workload", "C1"],
+                       capture_output=True, text=True, cwd=ROOT, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1 and json.loads(lines[0])["impl"] == "reference", r.stdout[-2000:]

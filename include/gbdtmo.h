@@ -257,6 +257,27 @@ gbdtmo_status gbdtmo_build_hist_packed(gbdtmo_ctx ctx, const gbdtmo_problem* p, 
                                        const uint8_t* bins, const uint8_t* packed, const int32_t* dflt,
                                        const int32_t* q, void* state, int64_t* hist, int32_t* cnt);
 
+/* Histograms from the paper's sparse storage (§3.2; NEXT-1), column-wise as the
+ * paper distributes the work: the same hist / cnt result as gbdtmo_build_hist
+ * (no default bins), built from the stored (non-zero) entries only:
+ *   hist[slot][f][c][b] = sum_{i in node, x_if stored, bin(i,f) = b != zbin[f]} q[i][c],  cnt likewise,
+ * then the zero bin of every feature (the implicit zeros and stored values binned with them) is
+ * filled in as node total - other bins (exact).  Work is proportional to nnz plus one pass over the
+ * built histograms.  All BUILD nodes of the level are zeroed and accumulated with global atomics
+ * (no shared-memory tiles, no root-count cache).
+ * col_ptr  int64 [m+1] (device), row_idx int32 [nnz] (device), nz_bins uint8 [nnz] (device: the bin
+ *          of each stored value, gbdtmo_csc_nz_bins), nnz = col_ptr[m] (host copy, sizes the grid)
+ * zbin     int32 [m] (device): bin of the value 0 per feature (gbdtmo_csc_nz_bins). */
+gbdtmo_status gbdtmo_build_hist_csc(gbdtmo_ctx ctx, const gbdtmo_problem* p, int32_t level, const int64_t* col_ptr,
+                                    const int32_t* row_idx, const uint8_t* nz_bins, int64_t nnz, const int32_t* zbin,
+                                    const int32_t* q, void* state, int64_t* hist, int32_t* cnt);
+/* Bins of the stored CSC values, gathered from the matrix gbdtmo_bin_csc wrote (nz_bins[e] =
+ * bins[row_idx[e] * ld_bins + f] for e in column f), and zbin[f] = bin(0) = #{cuts[f] <= 0} (R14).
+ * All pointers device; nz_bins uint8 [nnz] out, zbin int32 [m] out. */
+gbdtmo_status gbdtmo_csc_nz_bins(gbdtmo_ctx ctx, int32_t m, int32_t B, const int64_t* col_ptr, const int32_t* row_idx,
+                                 const uint8_t* bins, int64_t ld_bins, const float* cuts, uint8_t* nz_bins,
+                                 int32_t* zbin);
+
 /* ------------------------------------- (a)4 subtraction + (a)5 split search */
 
 /* For every active node of `level`:

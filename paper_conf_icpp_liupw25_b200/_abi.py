@@ -26,7 +26,7 @@ SYMBOLS = (
     "gbdtmo_find_split", "gbdtmo_split_record", "gbdtmo_partition", "gbdtmo_leaf_values",
     "gbdtmo_update_pred", "gbdtmo_tree_export", "gbdtmo_rows_export", "gbdtmo_default_bins", "gbdtmo_predict",
     "gbdtmo_set_option", "gbdtmo_search_small", "gbdtmo_bin_csc", "gbdtmo_packed_bins_bytes", "gbdtmo_pack_bins",
-    "gbdtmo_build_hist_packed", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
+    "gbdtmo_build_hist_packed", "gbdtmo_csc_nz_bins", "gbdtmo_build_hist_csc", "gbdtmo_peer_window_bytes", "gbdtmo_peer_open", "gbdtmo_peer_connect",
     "gbdtmo_peer_buffers", "gbdtmo_peer_status", "gbdtmo_peer_close", "gbdtmo_split_record_peer",
     "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async", "gbdtmo_bin_host",
     "gbdtmo_bin_host_workspace_bytes",
@@ -83,6 +83,8 @@ def lib():
             "gbdtmo_default_bins": ([P, P, i64, i32, i64, i32, i64, P], C.c_int),
             "gbdtmo_build_hist": ([P, PP, i32, P, P, P, P, P, P], C.c_int),
             "gbdtmo_build_hist_packed": ([P, PP, i32, P, P, P, P, P, P, P], C.c_int),
+            "gbdtmo_csc_nz_bins": ([P, i32, i32, P, P, P, i64, P, P, P], C.c_int),
+            "gbdtmo_build_hist_csc": ([P, PP, i32, P, P, P, i64, P, P, P, P, P], C.c_int),
             "gbdtmo_packed_bins_bytes": ([PP], sz),
             "gbdtmo_pack_bins": ([P, PP, P, P], C.c_int),
             "gbdtmo_find_split": ([P, PP, i32, P, P, P, P, P, P, P, P, P], C.c_int),
@@ -224,6 +226,15 @@ class Context:
         self._check(lib().gbdtmo_build_hist_packed(self._h, C.byref(p), level, _ptr(bins), _ptr(packed), _ptr(dflt),
                                                    _ptr(q), _ptr(state), _ptr(hist), _ptr(cnt)),
                     "gbdtmo_build_hist_packed")
+
+    def gbdtmo_csc_nz_bins(self, m, B, col_ptr, row_idx, bins, ld_bins, cuts, nz_bins, zbin):
+        self._check(lib().gbdtmo_csc_nz_bins(self._h, m, B, _ptr(col_ptr), _ptr(row_idx), _ptr(bins), ld_bins,
+                                             _ptr(cuts), _ptr(nz_bins), _ptr(zbin)), "gbdtmo_csc_nz_bins")
+
+    def gbdtmo_build_hist_csc(self, p, level, col_ptr, row_idx, nz_bins, nnz, zbin, q, state, hist, cnt):
+        self._check(lib().gbdtmo_build_hist_csc(self._h, C.byref(p), level, _ptr(col_ptr), _ptr(row_idx),
+                                                _ptr(nz_bins), nnz, _ptr(zbin), _ptr(q), _ptr(state), _ptr(hist),
+                                                _ptr(cnt)), "gbdtmo_build_hist_csc")
 
     @staticmethod
     def gbdtmo_packed_bins_bytes(p) -> int:

@@ -85,6 +85,14 @@ class Dataset:
     f_begin: int = 0
     m_global: int = 0
     dflt: Optional[torch.Tensor] = None   # int32 [m] default (most frequent) bin per feature
+    # CSC storage kept by bin_features_csc for gbdtmo_build_hist_csc: column
+    # pointers int64 [m+1], row indices int32 [nnz], bins of the stored values uint8 [nnz], bin of an
+    # implicit zero per feature int32 [m]
+    csc_col_ptr: Optional[torch.Tensor] = None
+    csc_row_idx: Optional[torch.Tensor] = None
+    csc_nz_bins: Optional[torch.Tensor] = None
+    csc_zbin: Optional[torch.Tensor] = None
+    csc_nnz: int = 0
 
 
 def bin_features(ctx: Context, X: torch.Tensor, B: int, f_begin: int = 0, m_global: Optional[int] = None,
@@ -157,7 +165,12 @@ def bin_features_csc(ctx: Context, values: torch.Tensor, row_idx: torch.Tensor, 
     ctx.gbdtmo_default_bins(bins, n, m, ld, B, max(1, n // 16), dflt)
     if not bool((dflt >= 0).any()):
         dflt = None
-    return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt)
+    nnz = int(cp_host[-1])
+    nz_bins = torch.empty(max(nnz, 1), dtype=torch.uint8, device=dev)
+    zbin = torch.empty(m, dtype=torch.int32, device=dev)
+    ctx.gbdtmo_csc_nz_bins(m, B, cp_dev, row_idx if nnz else None, bins, ld, cuts, nz_bins, zbin)
+    return Dataset(bins, nbins, cuts, n, m, ld, B, f_begin, m_global if m_global is not None else m, dflt,
+                   csc_col_ptr=cp_dev, csc_row_idx=row_idx, csc_nz_bins=nz_bins, csc_zbin=zbin, csc_nnz=nnz)
 
 
 class Booster:
@@ -168,11 +181,15 @@ class Booster:
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
                  small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
                  packed_bins: Optional[bool] = None, exchange: str = "collective", cache_root_counts: bool = True,
-                 fs_channel_groups: int = 0):
+                 fs_channel_groups: int = 0, csc_hist: Optional[bool] = None, csc_levels: Optional[int] = None):
         """exchange (only with `group`): "collective" = torch.distributed all-reduces per level;
         "peer" = the fused peer-memory exchange (NEXT-4, gbdtmo_*_peer): the keys / records are
         read from the other ranks' windows inside split_record / partition, no host collective.
-        fs_channel_groups: GBDTMO_OPT_FS_CHANNEL_GROUPS (0 automatic, 1 off, 2 / 4 / 8 forced)."""
+        fs_channel_groups: GBDTMO_OPT_FS_CHANNEL_GROUPS (0 automatic, 1 off, 2 / 4 / 8 forced).
+        csc_hist: build the histograms of levels < csc_levels (all by default) from the dataset's CSC
+        non-zeros (gbdtmo_build_hist_csc; datasets from bin_features_csc), the deeper ones from the bins;
+        None = automatic: on for CSC datasets below 4% density (measured crossover ~5%: C3 at 1% of its
+        entries 2.43 vs 4.36 ms per tree, at 20% 9.7 vs 4.6; profiles/r02c_csc_probe.jsonl)."""
         self.ctx, self.ds, self.params, self.group = ctx, ds, params, group
         assert exchange in ("collective", "peer")
         self.exchange = exchange if group is not None else "collective"
@@ -188,6 +205,16 @@ class Booster:
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
+        if csc_hist is None:
+            csc_hist = ds.csc_zbin is not None and ds.csc_nnz < 0.04 * ds.n * ds.m
+        self.csc_hist = bool(csc_hist)
+        self.csc_levels = params.D if csc_levels is None else int(csc_levels)
+        if self.csc_hist:
+            assert ds.csc_zbin is not None, "csc_hist needs a dataset from bin_features_csc"
+            cache_root_counts = False
+            if self.csc_levels >= params.D:      # no level reads the bins for histograms
+                self.gmem_max_rows = 0
+                packed_bins = False
         self.fs_channel_groups = int(fs_channel_groups)
         dev = ds.bins.device
         self.device = dev
@@ -317,7 +344,11 @@ class Booster:
         if time_hist:
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-        if self.packed is not None:
+        if self.csc_hist and lvl < self.csc_levels:
+            ds = self.ds
+            ctx.gbdtmo_build_hist_csc(p, lvl, ds.csc_col_ptr, ds.csc_row_idx, ds.csc_nz_bins, ds.csc_nnz, ds.csc_zbin,
+                                      self.q, self.state, self.hist[cur], self.cnt[cur])
+        elif self.packed is not None:
             ctx.gbdtmo_build_hist_packed(p, lvl, self.ds.bins, self.packed, self.dflt, self.q, self.state,
                                          self.hist[cur], self.cnt[cur])
         else:

@@ -259,7 +259,7 @@ k_find_split(gbdtmo_problem p, int level, const int32_t* __restrict__ nbins, con
 // Half-row variant (no default bins, 128 < B <= 256): two warps per (node, feature), lane l of
 // half h owns bins [128 h + 4 l, +4), so a lane holds half the row state of k_find_split and
 // the kernel runs at twice the occupancy (the 8-bin kernel is latency-bound at 128 registers:
-// ncu, profiles/r02_ncu_fs_c2.txt).  The halves need no exchange: half 0 prefix-sums its
+// ncu, profiles/r02_ncu_fs_C2.txt).  The halves need no exchange: half 0 prefix-sums its
 // bins (left sums), half 1 suffix-sums its bins (right sums, bins > b) and both complete the
 // other side from the exact node totals (node_sum = the sum of the node's histogram row in
 // int64), so every G_L, G_R, C_L is the same integer as in k_find_split and the gains and

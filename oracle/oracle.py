@@ -42,7 +42,8 @@ def build(force: bool = False) -> str:
 def lib():
     global _LIB
     if _LIB is None:
-        _LIB = C.CDLL(build())
+        # ORACLE_LIB: an instrumented build of the same source (tools/oracle_asan.sh), test infrastructure only
+        _LIB = C.CDLL(os.environ.get("ORACLE_LIB") or build())
         P = C.c_void_p
         i32, i64, f64 = C.c_int32, C.c_int64, C.c_double
         _LIB.oracle_bin.argtypes = [P, i64, i32, i64, i32, P, P, P]

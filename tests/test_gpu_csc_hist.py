@@ -81,3 +81,26 @@ def test_csc_histogram_trees_vs_oracle(orc, pkg, ctx, case, small, levels):
         sp = trees[t]["node_state"] == 1
         np.testing.assert_allclose(trees[t]["gain"][sp], ref["gain"][t][sp], rtol=1e-6)
     assert np.max(np.abs(b.pred.cpu().numpy() - ref["pred"])) <= 1e-4
+
+
+def test_csc_histogram_edge_cases(orc, pkg, ctx):
+    """No stored entries at all (every feature constant 0: the root stays a leaf, as in the oracle),
+    and one column holding every row (no implicit zeros) next to empty columns."""
+    w = dataclasses.replace(gen.WORKLOADS["C1"], B=16, T=2, D=3)
+    X0 = gen.features_host(w)
+    Y = gen.targets_host(w, X0)
+    for X in (np.zeros_like(X0), np.concatenate([X0[:, :1] + 10.0, np.zeros_like(X0[:, 1:])], axis=1)):
+        values, row_idx, col_ptr = orc.csc_from_dense(X)
+        ds = pkg.bin_features_csc(ctx, torch.from_numpy(values).to(DEV), torch.from_numpy(row_idx).to(DEV),
+                                  torch.from_numpy(col_ptr), X.shape[0], w.B)
+        cuts, nbins, bins = orc.bin_matrix(X, w.B)
+        ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                        lr=w.lr, min_node=w.min_node)
+        P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+        b = pkg.Booster(ctx, ds, torch.from_numpy(Y).to(DEV), P, csc_hist=True)
+        b.fit()
+        torch.cuda.synchronize()
+        for t in range(w.T):
+            assert not compare_trees(to_np(b.trees[t]), ref["state"][t], ref["feat"][t], ref["bin"][t],
+                                     ref["nrows"][t])
+        assert np.max(np.abs(b.pred.cpu().numpy() - ref["pred"])) <= 1e-4

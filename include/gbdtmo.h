@@ -117,10 +117,14 @@ const char*   gbdtmo_last_error(gbdtmo_ctx ctx);
  *     (fewer than 32 / CG warps per SM) splits every (node, feature)'s channel loop over CG = 2, 4
  *     or 8 warp pairs whose Eq. (3) partial sums are added in shared memory in a fixed order; 1:
  *     never; 2 / 4 / 8: always, with that CG (at most d).  Same (f, b) decisions up to near-ties;
- *     gains differ by fp64 summation order. */
+ *     gains differ by fp64 summation order.
+ *   GBDTMO_OPT_HIST_WAVES: histogram work items wanted per level, in multiples of the SM count
+ *     (a level's BUILD rows are cut into chunks so that chunks x tiles reaches it); 0 (default) = 2.
+ *     Fewer waves leave more nodes to a single chunk (sole-writer flushes, no zeroing); chosen per
+ *     shape by measurement (tools/calibrate_hist.py).  Same results. */
 enum { GBDTMO_OPT_GMEM_MAX_ROWS = 1, GBDTMO_OPT_SMALL_MAX_ROWS = 2, GBDTMO_OPT_HIST_KERNEL = 3,
        GBDTMO_OPT_PEER_TIMEOUT_MS = 4 /* bound of every peer-flag wait (gbdtmo_peer_*), default 30000 */,
-       GBDTMO_OPT_FS_CHANNEL_GROUPS = 5 };
+       GBDTMO_OPT_FS_CHANNEL_GROUPS = 5, GBDTMO_OPT_HIST_WAVES = 6 };
 gbdtmo_status gbdtmo_set_option(gbdtmo_ctx ctx, int32_t option, int64_t value);
 /* Cached root counts.  The root holds all n rows in every tree, so its count histogram
  * cnt[0][f][b] = #{i : bin(i, f) = b} (PAPER.md:214's histogram, count channel) is the same for

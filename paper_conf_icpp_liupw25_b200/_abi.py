@@ -31,7 +31,8 @@ SYMBOLS = (
     "gbdtmo_partition_peer", "gbdtmo_set_root_counts", "gbdtmo_peer_status_async", "gbdtmo_bin_host",
     "gbdtmo_bin_host_workspace_bytes",
 )
-OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS, OPT_FS_CHANNEL_GROUPS = 1, 2, 3, 4, 5
+(OPT_GMEM_MAX_ROWS, OPT_SMALL_MAX_ROWS, OPT_HIST_KERNEL, OPT_PEER_TIMEOUT_MS, OPT_FS_CHANNEL_GROUPS,
+ OPT_HIST_WAVES) = 1, 2, 3, 4, 5, 6
 PEER_HANDLE_BYTES = 64
 
 

@@ -181,7 +181,8 @@ class Booster:
                  sparse_default: bool = False, gmem_max_rows: Optional[int] = None,
                  small_max_rows: Optional[int] = None, hist_kernel: Optional[int] = None,
                  packed_bins: Optional[bool] = None, exchange: str = "collective", cache_root_counts: bool = True,
-                 fs_channel_groups: int = 0, csc_hist: Optional[bool] = None, csc_levels: Optional[int] = None):
+                 fs_channel_groups: int = 0, csc_hist: Optional[bool] = None, csc_levels: Optional[int] = None,
+                 hist_waves: Optional[int] = None):
         """exchange (only with `group`): "collective" = torch.distributed all-reduces per level;
         "peer" = the fused peer-memory exchange (NEXT-4, gbdtmo_*_peer): the keys / records are
         read from the other ranks' windows inside split_record / partition, no host collective.
@@ -202,6 +203,8 @@ class Booster:
         # shared-memory lane mapping: 0 row-pair tiles, 1 diagonal K = 4 tiles (measured per shape)
         self.hist_kernel = variant_threshold(V, ds.m, "hist_kernel", n=ds.n) if hist_kernel is None \
             else int(hist_kernel)
+        # histogram work items per level in SM multiples (GBDTMO_OPT_HIST_WAVES; measured per shape)
+        self.hist_waves = variant_threshold(V, ds.m, "hist_waves", n=ds.n) if hist_waves is None else int(hist_waves)
         # sparsity-aware default-bin skip; None = accumulate every bin.  Off by
         # default: measured slower on C2 (8.55 vs 7.84 ms/tree), where per-node overheads dominate.
         self.dflt = ds.dflt if sparse_default else None
@@ -388,6 +391,7 @@ class Booster:
         ctx.gbdtmo_set_option(_abi.OPT_SMALL_MAX_ROWS, self.small_max_rows)
         ctx.gbdtmo_set_option(_abi.OPT_HIST_KERNEL, self.hist_kernel)
         ctx.gbdtmo_set_option(_abi.OPT_FS_CHANNEL_GROUPS, self.fs_channel_groups)
+        ctx.gbdtmo_set_option(_abi.OPT_HIST_WAVES, self.hist_waves)
         ctx.gbdtmo_set_root_counts(self.root_cnt)
 
     def _mark(self, name: str, on: bool):

@@ -70,6 +70,10 @@ extern "C" gbdtmo_status gbdtmo_set_option(gbdtmo_ctx c, int32_t option, int64_t
       }
       ctx->fs_channel_groups = value;
       return GBDTMO_OK;
+    case GBDTMO_OPT_HIST_WAVES:
+      if (value < 0 || value > 64) { ctx->err = "gbdtmo_set_option: HIST_WAVES must be in [0, 64]"; return GBDTMO_EINVAL; }
+      ctx->hist_waves = value;
+      return GBDTMO_OK;
     default: ctx->err = "gbdtmo_set_option: unknown option"; return GBDTMO_EINVAL;
   }
 }

@@ -28,6 +28,7 @@ struct Ctx {
   int64_t hist_kernel = 0;     // GBDTMO_OPT_HIST_KERNEL: 0 row-pair (K <= 16), 1 diagonal (K = 4), 2 TMA-staged row-pair
   int64_t peer_timeout_ms = 30000;   // GBDTMO_OPT_PEER_TIMEOUT_MS: bound of every peer-flag wait
   int64_t fs_channel_groups = 0;     // GBDTMO_OPT_FS_CHANNEL_GROUPS: 0 automatic, 1 off, 2 / 4 forced
+  int64_t hist_waves = 0;            // GBDTMO_OPT_HIST_WAVES: histogram work items per level in SM multiples (0: default)
   Peer* peer = nullptr;        // gbdtmo_peer_open / _connect (peer.cu)
   const int32_t* root_cnt = nullptr;   // gbdtmo_set_root_counts: cached root counts [m][B] (or null)
   cudaStream_t copy_stream = nullptr;  // gbdtmo_bin_host: host -> device strip copies (created on first use)

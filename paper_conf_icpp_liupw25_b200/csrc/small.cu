@@ -317,7 +317,8 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
   }
 }
 
-bool small_supported(const gbdtmo_problem& p) { return p.B <= 256 && seg_cap(p) >= 64; }
+// (k_split_record's row pass for SMALL nodes covers at most 64 channels: d <= 32 softmax / 64 MSE)
+bool small_supported(const gbdtmo_problem& p) { return p.B <= 256 && channels(p) <= 64 && seg_cap(p) >= 64; }
 int64_t small_rows_cap(const gbdtmo_problem& p) { return seg_cap(p); }
 
 }  // namespace gbdtmo

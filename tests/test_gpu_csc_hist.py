@@ -70,7 +70,11 @@ def test_csc_histogram_trees_vs_oracle(orc, pkg, ctx, case, small, levels):
     torch.cuda.synchronize()
     trees = [to_np(t) for t in b.trees]
     for t in range(w.T):
-        if compare_trees(trees[t], ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]):
+        try:
+            differs = bool(compare_trees(trees[t], ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]))
+        except AssertionError:          # a different split moved rows
+            differs = True
+        if differs:
             pred, ties = tie_locked_oracle(orc, bins, nbins, w.B, y, w.loss, np.zeros_like(y), trees, 0, w.T, w.D,
                                            w.lam, w.gamma, w.lr, w.min_node)
             assert ties

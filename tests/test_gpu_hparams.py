@@ -82,6 +82,14 @@ def _run(orc, pkg, ctx, w, X, Y, lam, gamma_frac, lr, min_node, hk, **kw):
     return ref
 
 
+def _differs(tree, ref, t):
+    """True where tree t differs from the oracle's (a different split moves rows: compare_trees asserts)."""
+    try:
+        return bool(compare_trees(tree, ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]))
+    except AssertionError:
+        return True
+
+
 GRID = [
     # case, d, B, lambda, gamma_frac, lr, min_node
     ("C1", None, None, 0.0, 0.0, 1.0, 20),
@@ -134,7 +142,7 @@ def test_channel_split_search_vs_oracle(orc, pkg, ctx, case, d, lam, gfrac, mn, 
     torch.cuda.synchronize()
     trees = [to_np(t) for t in b.trees]
     for t in range(w.T):
-        if compare_trees(trees[t], ref["state"][t], ref["feat"][t], ref["bin"][t], ref["nrows"][t]):
+        if _differs(trees[t], ref, t):
             # a near-tie (min_node 1, binary softmax: symmetric candidates): the tie-locked oracle
             # (R30) adopts the GPU's choice where the gains tie within 1e-6 and must agree elsewhere
             pred, ties = tie_locked_oracle(orc, bins, nbins, w.B, y, w.loss, np.zeros_like(y), trees, 0, w.T,
@@ -193,3 +201,29 @@ def test_deep_trees_vs_oracle(orc, pkg, ctx, case, D):
     Y = gen.targets_host(w, X)
     ref = _run(orc, pkg, ctx, w, X, Y, 1.0, 0.0, 1.0, 5, 0)
     assert np.any(ref["state"][:, (1 << (D - 1)) - 1:(1 << D) - 1] == 1)      # splits at the last level
+
+
+def test_small_option_ignored_beyond_64_channels(orc, pkg, ctx):
+    """GBDTMO_OPT_SMALL_MAX_ROWS on a softmax problem with 2 x 40 channels: the small-node path (its
+    split records cover at most 64 channels) must stay off, and the trees equal the oracle's."""
+    w = gen.sweep(40, n=4_000, m=16, T=2, D=4)
+    X = gen.features_host(w)
+    Y = gen.targets_host(w, X)
+    cuts, nbins, bins = orc.bin_matrix(X, w.B)
+    ref = orc.train(bins, nbins, w.B, Y.astype(np.float64), loss=w.loss, T=w.T, D=w.D, lam=w.lam, gamma=w.gamma,
+                    lr=w.lr, min_node=w.min_node)
+    P = pkg.Params(loss=w.loss, T=w.T, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr, min_node=w.min_node)
+    b = pkg.Booster(ctx, pkg.bin_features(ctx, torch.from_numpy(X).cuda(), w.B), torch.from_numpy(Y).cuda(), P,
+                    small_max_rows=2000)
+    b.fit()
+    torch.cuda.synchronize()
+    trees = [to_np(t) for t in b.trees]
+    if any(_differs(trees[t], ref, t) for t in range(w.T)):
+        # near-ties among 40 classes' Eq. (3) sums: the tie-locked oracle (R30) must accept every difference
+        y = Y.astype(np.float64)
+        pred, ties = tie_locked_oracle(orc, bins, nbins, w.B, y, w.loss, np.zeros_like(y), trees, 0, w.T, w.D,
+                                       w.lam, w.gamma, w.lr, w.min_node)
+        assert ties
+        assert np.max(np.abs(b.pred.cpu().numpy() - pred)) <= 1e-4
+        return
+    assert np.max(np.abs(b.pred.cpu().numpy() - ref["pred"])) <= 1e-4

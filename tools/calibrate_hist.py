@@ -24,10 +24,14 @@ CANDIDATES = [0, 256, 512, 1024, 2048, 4096, 8192, 16384]
 SMALL_CANDIDATES = [0, 128, 256, 384, 512, 768, 1024, 1536, 2048, 4096]
 
 
-def time_trees(ctx, ds, Y, w, thr, small=0, warm=2, timed=3, hk=0):
+WAVES_CANDIDATES = [1, 2, 4]
+
+
+def time_trees(ctx, ds, Y, w, thr, small=0, warm=2, timed=3, hk=0, waves=0):
     P = pkg.Params(loss=w.loss, T=warm + timed, D=w.D, B=w.B, lam=w.lam, gamma=w.gamma, lr=w.lr,
                    min_node=w.min_node)
-    b = pkg.Booster(ctx, ds, Y, P, keep_model=False, gmem_max_rows=thr, small_max_rows=small, hist_kernel=hk)
+    b = pkg.Booster(ctx, ds, Y, P, keep_model=False, gmem_max_rows=thr, small_max_rows=small, hist_kernel=hk,
+                    hist_waves=waves)
     for _ in range(warm):
         b.step()
     torch.cuda.synchronize()
@@ -57,18 +61,24 @@ def main():
         # shared-memory lane mapping first (0 row-pair tiles, 1 diagonal K = 4 tiles), then thresholds
         rk = {k: time_trees(ctx, ds, Y, w, 0, 0, hk=k) for k in (0, 1)}
         hk = 1 if rk[1] < 0.98 * rk[0] else 0
-        res = {c: time_trees(ctx, ds, Y, w, c, hk=hk) for c in CANDIDATES}
+        # work items per level (GBDTMO_OPT_HIST_WAVES), default 2 unless another is >= 2% faster
+        rw = {k: time_trees(ctx, ds, Y, w, 0, 0, hk=hk, waves=k) for k in WAVES_CANDIDATES}
+        wv = min(rw, key=rw.get)
+        if rw[wv] > 0.98 * rw[2]:
+            wv = 2
+        res = {c: time_trees(ctx, ds, Y, w, c, hk=hk, waves=wv) for c in CANDIDATES}
         best = min(res, key=res.get)
         if res[best] > 0.98 * res[0]:          # noise guard: keep the default unless >= 2% faster
             best = 0
-        small_ok = w.d <= 32
-        rs = {c: time_trees(ctx, ds, Y, w, best, c, hk=hk) for c in (SMALL_CANDIDATES if small_ok else [0])}
+        small_ok = w.d * (2 if w.loss == gen.LOSS_SOFTMAX else 1) <= 64
+        rs = {c: time_trees(ctx, ds, Y, w, best, c, hk=hk, waves=wv) for c in (SMALL_CANDIDATES if small_ok else [0])}
         best_s = min(rs, key=rs.get)
         if rs[best_s] > 0.98 * rs[0]:
             best_s = 0
         entries.append({"workload": w.name, "V": V, "m": w.m, "n": w.n, "gmem_max_rows": best,
-                        "small_max_rows": best_s, "hist_kernel": hk,
+                        "small_max_rows": best_s, "hist_kernel": hk, "hist_waves": wv,
                         "ms_per_tree_kernel": {str(k): round(v, 4) for k, v in rk.items()},
+                        "ms_per_tree_waves": {str(k): round(v, 4) for k, v in rw.items()},
                         "ms_per_tree": {str(k): round(v, 4) for k, v in res.items()},
                         "ms_per_tree_small": {str(k): round(v, 4) for k, v in rs.items()}})
         print(json.dumps(entries[-1]), flush=True)

@@ -1,7 +1,9 @@
 // hist_csc.cu — (a)3 on the paper's sparse storage (§3.2 "Sparsity-aware data
-// storage"; NEXT-1): histograms built from the CSC non-zeros only, column-wise as the paper
-// distributes the work ("each GPU thread block is responsible for ... attribute
-// columns; warps process different training instances of these columns").
+// storage"; NEXT-1): histograms built from the CSC non-zeros only.  The paper gives each thread
+// block one or more attribute columns; here the column-major entries are spread
+// evenly instead (one thread per stored entry, its column by a binary search of col_ptr), since
+// column lengths vary by orders of magnitude in sparse data (a block-per-column variant was
+// latency-bound and slower: DESIGN.md §7, "CSC-driven histograms").
 //
 //   hist[slot][f][c][b] = sum_{i in node, x_if != 0, bin(i,f) = b, b != z_f} q[i][c]   (exact int64)
 //   cnt [slot][f][b]    = #{...}

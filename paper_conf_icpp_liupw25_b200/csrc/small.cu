@@ -36,8 +36,10 @@ constexpr int kSegCand = 256;          // candidates per (node, feature) <= dist
 struct SegLayout {
   int rc, V;
   int o_qs, o_warps, warp_bytes, bytes;
-  // per warp: cnt[256] u32 | candG[256] i64 | aux[256] (softmax candH i64 / MSE accR f64) |
-  //           acc[256] f64 | cpos[256] u16 | cbin[256] u8 | bk[rc] u8 | sb[rc + 8] u8 | sidxT[rc32] u16
+  // per warp: candG[256] i64 (bk[rc] u8 during the sort) | aux[256] (softmax candH i64 / MSE accR f64) |
+  //           acc[256] f64 (cnt[256] u32 during the sort) | cpos[256] u16 | cbin[256] u8 | sb[rc + 16] u8 |
+  //           sidxT[rc32] u16.  cnt and bk are dead once the rows are scattered in bin order, before
+  //           the candidate arrays are written, so they share space with acc and candG.
   int o_cnt, o_candG, o_aux, o_acc, o_cpos, o_cbin, o_bk, o_sb, o_sidx;
 };
 
@@ -47,14 +49,14 @@ __host__ __device__ inline SegLayout seg_layout(const gbdtmo_problem& p, int64_t
   L.V = channels(p);
   L.o_qs = 4 * L.rc;
   L.o_warps = (L.o_qs + 4 * L.V * L.rc + 15) / 16 * 16;
-  L.o_cnt = 0;
-  L.o_candG = L.o_cnt + 4 * 256;
+  L.o_candG = 0;
+  L.o_bk = L.o_candG;                                // (rc <= 1024 <= 8 kSegCand bytes)
   L.o_aux = L.o_candG + 8 * kSegCand;
   L.o_acc = L.o_aux + 8 * kSegCand;
+  L.o_cnt = L.o_acc;                                 // 4 x 256 <= 8 kSegCand bytes
   L.o_cpos = L.o_acc + 8 * kSegCand;
   L.o_cbin = L.o_cpos + 2 * kSegCand;
-  L.o_bk = L.o_cbin + kSegCand;
-  L.o_sb = L.o_bk + L.rc;
+  L.o_sb = L.o_cbin + kSegCand;
   L.o_sidx = L.o_sb + L.rc + 16;
   L.warp_bytes = (L.o_sidx + 2 * L.rc + 15) / 16 * 16;
   L.bytes = L.o_warps + kSegWarps * L.warp_bytes;
@@ -63,9 +65,9 @@ __host__ __device__ inline SegLayout seg_layout(const gbdtmo_problem& p, int64_t
 
 __host__ __device__ inline int64_t seg_cap(const gbdtmo_problem& p) {
   const int V = channels(p);
-  // bytes(rc) = 4 rc (1 + V) + W (7936 + 4 rc + 16) (+ alignment)
-  const int64_t fixed = (int64_t)kSegWarps * (4 * 256 + 3 * 8 * kSegCand + 2 * kSegCand + kSegCand + 16) + 64;
-  int64_t r = (kHistSmemBudget - fixed) / (4 * (1 + V) + 4 * kSegWarps);
+  // bytes(rc) = 4 rc (1 + V) + W (6912 + 3 rc + 16) (+ alignment)
+  const int64_t fixed = (int64_t)kSegWarps * (3 * 8 * kSegCand + 2 * kSegCand + kSegCand + 16 + 16) + 64;
+  int64_t r = (kHistSmemBudget - fixed) / (4 * (1 + V) + 3 * kSegWarps);
   r = r / 32 * 32;
   if (r > 1024) r = 1024;                          // <= 32 positions per lane (one candidate bit each)
   return r < 0 ? 0 : r;
@@ -343,10 +345,13 @@ extern "C" gbdtmo_status gbdtmo_search_small(gbdtmo_ctx c, const gbdtmo_problem*
   const int64_t LN = int64_t(1) << level;
   const bool sm = p->loss == GBDTMO_LOSS_SOFTMAX;
   const SegLayout L = seg_layout(*p, rcap);
-  // feature blocks per node: ~8 waves of resident CTAs over the level's (at most LN) small nodes,
+  // feature blocks per node: GBDTMO_SEG_WAVES waves of resident CTAs over the level's (at most LN) small nodes,
   // so nodes of different sizes balance (ncu at 2.6 waves: 46% issue, idle SMs in the tail)
   const int per_sm = (int)((ctx->max_smem_optin) / (L.bytes + 1024));
-  int64_t fb = (8LL * ctx->num_sms * (per_sm < 1 ? 1 : per_sm) + LN - 1) / LN;
+#ifndef GBDTMO_SEG_WAVES
+#define GBDTMO_SEG_WAVES 32   // waves of (node, feature block) CTAs: C2 4.28 / 4.23 / 4.20 / 4.20 ms per tree at 8 / 16 / 32 / 64
+#endif
+  int64_t fb = ((int64_t)GBDTMO_SEG_WAVES * ctx->num_sms * (per_sm < 1 ? 1 : per_sm) + LN - 1) / LN;
   const int64_t fb_max = (p->m + kSegWarps - 1) / kSegWarps;
   if (fb > fb_max) fb = fb_max;
   if (fb < 1) fb = 1;

@@ -31,6 +31,10 @@ namespace gbdtmo {
 #endif
 #define SEG_CHECK(cond) do { if (GBDTMO_BOUNDS_CHECK && !(cond)) __trap(); } while (0)
 constexpr int kSegWarps = 16;
+#ifndef GBDTMO_SEG_ILP
+#define GBDTMO_SEG_ILP 4
+#endif
+constexpr int kSegILP = GBDTMO_SEG_ILP;   // row loads in flight per lane in the per-output walk
 constexpr int kSegCand = 256;          // candidates per (node, feature) <= distinct bins - 1 <= 255
 
 struct SegLayout {
@@ -229,10 +233,10 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
       long long g = 0, hh = 0;
       int ci = cb;
       const int pe = min(PL, R - p0);              // this lane's positions
-      for (int i0 = 0; i0 < pe; i0 += 4) {         // 4 independent row loads in flight
-        int qg[4], qh[4];
+      for (int i0 = 0; i0 < pe; i0 += kSegILP) {   // kSegILP independent row loads in flight
+        int qg[kSegILP], qh[kSegILP];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < kSegILP; ++u) {
           const int r = i0 + u < pe ? (int)sidxT[(i0 + u) * 32 + lane] : -1;
           SEG_CHECK(r < R);
           if (SOFTMAX) {
@@ -245,7 +249,7 @@ k_seg_search(gbdtmo_problem p, int level, int rcap, const uint8_t* __restrict__ 
           }
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < kSegILP; ++u) {
           g += qg[u];
           if (SOFTMAX) hh += qh[u];
           if ((cm >> (i0 + u)) & 1u) {

@@ -19,6 +19,9 @@ constexpr int kFsWarps = 8;      // warps per block = features of one node per b
 #ifndef GBDTMO_FS_SOFTMAX_MINB
 #define GBDTMO_FS_SOFTMAX_MINB 4  // resident blocks per SM of the softmax half-row search: 4 (64 registers, 24 B spilled): C2 find_split 1.80 -> 1.70 ms (profiles/r02_ab_fs_softmax_minb4.jsonl)
 #endif
+#ifndef GBDTMO_REC_TRANSPOSE
+#define GBDTMO_REC_TRANSPOSE 1   // SMALL nodes' split records: rows' q through a shared tile (0: serial per left row)
+#endif
 #ifndef GBDTMO_FS_CG_OFF
 #define GBDTMO_FS_CG_OFF 0       // (A/B) 1: no channel-split search (k_find_split_c)
 #endif
@@ -723,6 +726,7 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
     if (blockIdx.y != 0) return;                  // (d <= 32: one block covers every channel)
     // one pass: warps take 32 rows at a time, lanes = channels sum the rows that go left
     __shared__ long long acc[2 * 32 + 1];
+    __shared__ int32_t tq[GBDTMO_REC_TRANSPOSE ? 8 : 1][32][33];
     for (int c = threadIdx.x; c <= V; c += blockDim.x) acc[c] = 0;
     __syncthreads();
     const int32_t* rl = (level & 1) ? s.rows1 : s.rows0;
@@ -732,14 +736,31 @@ __global__ void k_split_record(gbdtmo_problem p, int level, const int32_t* __res
       const int pos = pos0 + lane;
       const int r = pos < nb1 ? (level > 0 ? rl[pos] : pos) : -1;
       const bool left = r >= 0 && bins[(int64_t)r * p.ld_bins + fl] <= b;
-      unsigned msk = __ballot_sync(0xffffffffu, left);
+      const unsigned msk = __ballot_sync(0xffffffffu, left);
       nleft += __popc(msk);
-      while (msk) {
-        const int src = __ffs(msk) - 1;
-        msk &= msk - 1;
-        const int64_t rr = (int64_t)__shfl_sync(0xffffffffu, r, src) * V;
-        if (lane < V) a0 += q[rr + lane];
-        if (lane + 32 < V) a1 += q[rr + lane + 32];
+      if (GBDTMO_REC_TRANSPOSE) {
+        // lanes = rows: each left row's q values go through a [32][33] shared tile (independent
+        // loads, no per-row serial chain), then lanes = channels add the 32 rows
+        for (int cc = 0; cc < V; cc += 32) {
+#pragma unroll 8
+          for (int c = 0; c < 32; ++c)
+            tq[warp][lane][c] = (left && cc + c < V) ? q[(int64_t)r * V + cc + c] : 0;
+          __syncwarp();
+          long long sacc = 0;
+#pragma unroll 8
+          for (int i = 0; i < 32; ++i) sacc += tq[warp][i][lane];
+          if (cc == 0) a0 += sacc; else a1 += sacc;
+          __syncwarp();
+        }
+      } else {
+        unsigned mm = msk;
+        while (mm) {
+          const int src = __ffs(mm) - 1;
+          mm &= mm - 1;
+          const int64_t rr = (int64_t)__shfl_sync(0xffffffffu, r, src) * V;
+          if (lane < V) a0 += q[rr + lane];
+          if (lane + 32 < V) a1 += q[rr + lane + 32];
+        }
       }
     }
     if (lane < V) atomicAdd((unsigned long long*)&acc[lane], (unsigned long long)a0);

@@ -44,8 +44,7 @@ k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict_
     const int64_t* S = s.node_sum + h * (V + 1);
     int64_t* SL = s.node_sum + hl * (V + 1);
     int64_t* SR = s.node_sum + hr * (V + 1);
-    for (int c = 0; c < V; ++c) { SL[c] = rec[c]; SR[c] = S[c] - rec[c]; }
-    SL[V] = nl; SR[V] = S[V] - nl;
+    SL[V] = nl; SR[V] = S[V] - nl;                  // (the V channel sums: block-wide loop below)
     const bool deeper = level + 1 < p.D;
     const int64_t nr = (e - b) - nl;
     const bool al = deeper && nl >= 2 * (int64_t)p.min_node;
@@ -63,6 +62,19 @@ k_apply_records(gbdtmo_problem p, int level, State s, const int64_t* __restrict_
     else if (as) { ms = MODE_BUILD; }
     s.node_mode[hs] = ms;
     s.node_mode[hg] = mg;
+  }
+  __syncthreads();
+  // children's exact channel sums, spread over the block (one thread per node and channel: with
+  // V = 2 x 983 channels a per-node loop was ~0.2 ms per level)
+  for (int64_t e = threadIdx.x; e < LN * V; e += blockDim.x) {
+    const int64_t i = e / V;
+    const int c = (int)(e - i * V);
+    const int64_t h = first + i;
+    if (s.node_state[h] != GBDTMO_NODE_SPLIT) continue;
+    const int64_t* rec = xchg + i * RW;
+    const int64_t S = s.node_sum[h * (V + 1) + c];
+    s.node_sum[(2 * h + 1) * (V + 1) + c] = rec[c];
+    s.node_sum[(2 * h + 2) * (V + 1) + c] = S - rec[c];
   }
   __syncthreads();
   plan_level_chunks(p, s, level + 1, target_chunks, gmem_max_rows);
